@@ -1,0 +1,198 @@
+/*
+ * pm.h -- C-ABI of the B200 (sm_100a) photomosaic hot path
+ * (Yang, Ito & Nakano, "Photomosaic Generation by Rearranging Subimages,
+ * with GPU Acceleration", IPDPS workshops 2017).  Library: libpm.so.
+ *
+ * "P:<n>" cites line n of the paper text; "reading Rk" cites DESIGN.md's list
+ * of readings where the paper is silent or garbled.
+ *
+ * Conventions for every entry point
+ *   - d_* : device pointer on the CURRENT CUDA device; h_* : host pointer.
+ *   - stream : a cudaStream_t (NULL = legacy default stream).  Device work is
+ *     enqueued on it; functions that return host scalars synchronise it.
+ *   - Ownership: the caller allocates and frees every buffer it passes.  The
+ *     library keeps no state between calls except cached, immutable launch
+ *     plans; scratch memory comes from cudaMallocAsync on `stream` and is
+ *     freed before return.
+ *   - Errors: every argument is validated before any launch
+ *     (PM_ERR_INVALID, nothing enqueued).  CUDA failures map to PM_ERR_CUDA.
+ *     No C++ exception crosses this boundary.  Outputs are undefined on error.
+ *   - There is no CPU fallback: every step runs in this library's kernels.
+ *   - Thread-safe across distinct streams.
+ *   - All arithmetic is integer: results are bit-exact by construction.
+ */
+#ifndef PM_H_
+#define PM_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+struct CUstream_st;                       /* = cudaStream_t */
+typedef struct CUstream_st* pm_stream_t;
+
+typedef enum {
+  PM_OK = 0,
+  PM_ERR_INVALID = 1,        /* bad argument; nothing was launched            */
+  PM_ERR_CUDA = 2,           /* a CUDA runtime call or launch failed          */
+  PM_ERR_NOT_CONVERGED = 3,  /* max_rounds reached before a zero-swap round   */
+  PM_ERR_UNSUPPORTED = 4,    /* valid, but outside what this build supports   */
+  PM_ERR_NOT_PERMUTATION = 5 /* d_perm is not a bijection of [0, S)    */
+} pm_status_t;
+
+/* Local-search implementation selector for pm_local_search_ex. */
+typedef enum {
+  PM_LS_AUTO = 0,      /* pick the fastest method supported for S            */
+  PM_LS_CLASS = 1,     /* one kernel per colour class P_i, the paper's own
+                          launch structure, replayed as a CUDA graph  */
+  PM_LS_CTA = 2,       /* one CTA runs every round on the device: r and the
+                          maintained diagonal d in shared memory, E gathered
+                          from L2/HBM (S <= pm_ls_cta_max_S())                */
+  PM_LS_WINDOW = 3     /* one CTA, plus a shared-memory window of each slot's
+                          upcoming E entries streamed ahead of the classes    */
+} pm_ls_method_t;
+
+const char* pm_status_string(pm_status_t s);
+
+/* Packed tile stride in bytes: P = M*M*C rounded up to a multiple of 64
+ * (the zero padding adds |0-0| = 0 to every E entry). */
+int64_t pm_tile_stride(int32_t M, int32_t C);
+
+/* Step 1: cut an N x N image into S = (N/M)^2 tiles of M x M.
+ *   d_img   : u8 [N][N][C], row-major HWC, no padding (reading R2).
+ *   d_tiles : u8 [S][ld_tiles], ld_tiles >= pm_tile_stride(M, C), multiple of
+ *             16.  Tile u = grid cell (u / (N/M), u % (N/M)) (raster, reading
+ *             R4); bytes in (y, x, c) order; bytes [M*M*C, ld_tiles) zeroed.
+ * Async on stream.  PM_ERR_INVALID unless N % M == 0, M >= 1, C >= 1. */
+pm_status_t pm_pack_tiles(const uint8_t* d_img, int32_t N, int32_t M, int32_t C,
+                          uint8_t* d_tiles, int64_t ld_tiles, pm_stream_t stream);
+
+/* Step 2, Eq. (1):
+ *   E[(u - row_begin) * ld_E + v] = sum_{y,x < M, c < C} |I_u(y,x,c) - T_v(y,x,c)|
+ * for input tiles u in [row_begin, row_end) and every target tile v in
+ * [0, S), S = (N/M)^2 -- the weight w_{u,v} of P:94 (rows = input tiles).
+ *   d_input, d_target : u8 [N][N][C] HWC images (as pm_pack_tiles).
+ *   d_E : int32, (row_end - row_begin) rows of ld_E >= S entries.
+ * Requires 255*M*M*C <= INT32_MAX (reading R11).  Async on stream (packs both
+ * images into scratch tiles, then runs the VABSDIFF4 SAD kernel). */
+pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target,
+                            int32_t N, int32_t M, int32_t C,
+                            int32_t row_begin, int32_t row_end,
+                            int32_t* d_E, int64_t ld_E, pm_stream_t stream);
+
+/* Step 2 on already-packed tiles (pm_pack_tiles layout, same ld_tiles for
+ * both), for callers that keep the tiles resident:
+ *   E[(u - row_begin) * ld_E + v] = sum_{k < P} |Itiles[u][k] - Ttiles[v][k]|,
+ * u in [row_begin, row_end), v in [0, S).  P = M*M*C; bytes P..ld_tiles-1
+ * must be zero in both (pm_pack_tiles guarantees it).  Async on stream. */
+pm_status_t pm_error_matrix_tiles(const uint8_t* d_input_tiles, const uint8_t* d_target_tiles,
+                                  int64_t ld_tiles, int32_t S, int32_t P,
+                                  int32_t row_begin, int32_t row_end,
+                                  int32_t* d_E, int64_t ld_E, pm_stream_t stream);
+
+/* Theorem 1: number of non-empty edge groups of K_S:
+ * S - 1 for even S, S for odd S, 0 for S < 2. */
+int32_t pm_num_colors(int32_t S);
+
+/* Edge groups P_{class_begin+1} .. P_{class_end}, 0-indexed slots,
+ * in the paper's group order and, inside a group, by increasing smaller index
+ * (exactly the printed K_16 table for S = 16).  Host-side, for tests and
+ * inspection; the kernels generate the same groups on the fly (reading R7:
+ * pairs u + v == 2i + 1 (mod m), m = S-1 for even S, m = S for odd S; the
+ * fixed point joins vertex S when S is even and idles when S is odd).
+ *   h_pairs : int32 [class_end - class_begin][S/2][2], each (u, v) with u < v;
+ *             for odd S the last entry of every group is (-1, -1). */
+pm_status_t pm_edge_coloring(int32_t S, int32_t class_begin, int32_t class_end, int32_t* h_pairs);
+
+/* Step 3, Algorithm 2: parallel 2-swap local search over the
+ * edge groups, groups in order i = 1..S, all pairs of a group concurrently,
+ * rounds repeated until a round performs no swap.  Slot-indexed (reading R5):
+ * for each pair (u, v) of the group, with a = r[u], b = r[v],
+ *   if E[a][u] + E[b][v] > E[b][u] + E[a][v]   (strict, reading R6)
+ *   then r[u] = b, r[v] = a.
+ *   d_E    : int32 [S][ld_E] from pm_error_matrix (rows = input tiles).
+ *   d_perm : int32 [S]; in: the initial rearrangement (identity per the
+ *            paper, reading R7; any bijection resumes exactly), out: final r.
+ *            r[u] = input tile placed at target slot u (Eq. 2's r).
+ *   max_rounds : 0 = until convergence; else stop after that many rounds and
+ *            return PM_ERR_NOT_CONVERGED (d_perm then holds the state after
+ *            the last full round, so calling again resumes bit-identically).
+ *   h_rounds : rounds executed, counting the final zero-swap round (R10).
+ *   h_swaps  : total swaps.
+ * Synchronises `stream`.  PM_ERR_NOT_PERMUTATION if d_perm is not a
+ * bijection (checked on the device before any swap). */
+pm_status_t pm_local_search(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                            int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
+                            pm_stream_t stream);
+
+/* pm_local_search with an explicit method (pm_ls_method_t) and an optional
+ * per-round swap log h_swaps_per_round[0 .. min(rounds, len)-1] (may be NULL). */
+pm_status_t pm_local_search_ex(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                               int32_t max_rounds, int32_t method,
+                               int32_t* h_rounds, int64_t* h_swaps,
+                               int64_t* h_swaps_per_round, int32_t len,
+                               pm_stream_t stream);
+
+/* Algorithm 2 without any host synchronisation (for pipelines and graphs):
+ * as pm_local_search, but the outcome is written to DEVICE memory
+ *   d_result : int64 [3] = {status (pm_status_t), rounds, swaps}
+ * when the enqueued work completes.  The return value only reports argument
+ * and launch errors. */
+pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                  int32_t max_rounds, int32_t method, int64_t* d_result,
+                                  pm_stream_t stream);
+
+/* Largest S the single-CTA methods accept on this device (shared-memory
+ * bound); 0 if no device. */
+int32_t pm_ls_cta_max_S(void);
+
+/* r := identity (Alg. 1/2 start from the input image as given, P:116-120,
+ * reading R7).  d_perm : int32 [S].  Async on stream. */
+pm_status_t pm_init_identity(int32_t* d_perm, int32_t S, pm_stream_t stream);
+
+/* Eq. (2): *h_cost = sum_u E[r[u]][u] (int64, reading R11).
+ * Synchronises `stream`. */
+pm_status_t pm_cost(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm,
+                    int64_t* h_cost, pm_stream_t stream);
+
+/* Eq. (2) without the host sync: d_cost (int64 [1], device) is overwritten. */
+pm_status_t pm_cost_async(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm,
+                          int64_t* d_cost, pm_stream_t stream);
+
+/* The whole approximation pipeline of Sec. V in one call, on
+ * device buffers: Step 1 + Step 2 into d_E (caller-owned, [S][ld_E]), r :=
+ * identity, Algorithm 2 (method as pm_local_search_ex), Eq. (2).
+ * Outputs d_perm (int32 [S]) and the host scalars.  Synchronises `stream`. */
+pm_status_t pm_photomosaic(const uint8_t* d_input, const uint8_t* d_target,
+                           int32_t N, int32_t M, int32_t C,
+                           int32_t* d_E, int64_t ld_E, int32_t* d_perm, int32_t method,
+                           int32_t* h_rounds, int64_t* h_swaps, int64_t* h_cost,
+                           pm_stream_t stream);
+
+/* pm_photomosaic without any host synchronisation: d_result (int64 [4],
+ * device) receives {status, rounds, swaps, cost} when the work completes. */
+pm_status_t pm_photomosaic_async(const uint8_t* d_input, const uint8_t* d_target,
+                                 int32_t N, int32_t M, int32_t C,
+                                 int32_t* d_E, int64_t ld_E, int32_t* d_perm, int32_t method,
+                                 int64_t* d_result, pm_stream_t stream);
+
+/* Same pipeline from HOST images to HOST results (the end-to-end call):
+ * copies h_input / h_target (u8 [N][N][C]) to the device, runs
+ * pm_photomosaic with library-owned scratch, copies r back to h_perm
+ * (int32 [S]).  Pinned host memory gives full PCIe/C2C bandwidth; pageable
+ * memory works but is slower.  Synchronises `stream`. */
+pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
+                                int32_t N, int32_t M, int32_t C, int32_t method,
+                                int32_t* h_perm, int32_t* h_rounds, int64_t* h_swaps,
+                                int64_t* h_cost, pm_stream_t stream);
+
+/* Number of this library's kernel launches enqueued by the calling process
+ * so far (for launch accounting in benchmarks). */
+int64_t pm_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PM_H_ */

@@ -1,0 +1,243 @@
+// k_sad.cu -- Step 1 (tile packing) and Step 2 (the all-pairs tile
+// error matrix, Eq. 1) for sm_100a.
+//
+// Eq. (1) is an L1 / sum-of-absolute-differences metric (reading R1), which is
+// not bilinear, so it does not map onto tcgen05 tensor cores (the exact
+// threshold-decomposition form would need 255x the MACs; DESIGN.md "E
+// kernel").  It runs on the integer ALU pipe instead: one
+// `vabsdiff4.u32.u32.u32.add` (SASS VABSDIFF4.U8.ACC) consumes 4 byte pairs
+// and accumulates into an int32, and issues at the IADD3 rate (64/clk/SM,
+// tools/ubench_alu.cu).  The kernel is a register-blocked "SAD-GEMM":
+//   * CTA tile 128 (input tiles u) x 128 (target tiles v), 256 threads, each
+//     thread 8 x 8 outputs (rows ty + 16 i, cols tx + 16 j -> conflict-free
+//     LDS.128 on a 80-byte padded smem row stride);
+//   * K (the P bytes of a tile) streamed in 64-byte chunks through a 4-stage
+//     cp.async.cg ring (16-byte copies, L2-only), so smem holds 16 words per
+//     row per stage;
+//   * per 4 K-words a thread issues 16 LDS.128 and 256 VABSDIFF4 (16:1);
+//   * split-K over gridDim.z for small S (integer red.add is exact and
+//     order-independent), chosen on the host to fill all 148 SMs.
+#include "pm_internal.cuh"
+
+namespace pm {
+
+// ---------------------------------------------------------------- Step 1 ---
+// One thread per 4 output bytes of the packed layout; tile t in
+// [tile_begin, tile_end) goes to row t - tile_begin of `tiles`.
+__global__ void k_pack(const uint8_t* __restrict__ img, int32_t N, int32_t M, int32_t C,
+                       uint8_t* __restrict__ tiles, int64_t ld_tiles, int32_t tile_begin,
+                       int32_t tile_end) {
+  const int32_t g = N / M;
+  const int32_t P = M * M * C;
+  const int64_t words_per_tile = ld_tiles / 4;
+  const int64_t total = (int64_t)(tile_end - tile_begin) * words_per_tile;
+  for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < total;
+       w += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t t = tile_begin + w / words_per_tile;
+    const int32_t k0 = (int32_t)(w % words_per_tile) * 4;
+    const int64_t ty = t / g, tx = t % g;
+    uint32_t out = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int32_t k = k0 + q;
+      uint32_t byte = 0;
+      if (k < P) {
+        const int32_t pix = k / C, c = k - pix * C;
+        const int32_t y = pix / M, x = pix - y * M;
+        byte = img[((ty * M + y) * (int64_t)N + tx * M + x) * C + c];
+      }
+      out |= byte << (8 * q);
+    }
+    reinterpret_cast<uint32_t*>(tiles + (t - tile_begin) * ld_tiles)[k0 / 4] = out;
+  }
+}
+
+cudaError_t launch_pack(const uint8_t* img, int32_t N, int32_t M, int32_t C, uint8_t* tiles,
+                        int64_t ld_tiles, int32_t tile_begin, int32_t tile_end, cudaStream_t st) {
+  const int64_t total = (int64_t)(tile_end - tile_begin) * (ld_tiles / 4);
+  if (total <= 0) return cudaSuccess;
+  int64_t blocks = (total + 255) / 256;
+  if (blocks > 148 * 16) blocks = 148 * 16;
+  k_pack<<<(unsigned)blocks, 256, 0, st>>>(img, N, M, C, tiles, ld_tiles, tile_begin, tile_end);
+  note_launch();
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------- Step 2 ---
+namespace sad {
+constexpr int kThreads = 256;
+constexpr int BM = 128, BN = 128;
+constexpr int BKW = 16;          // K words (4 bytes each) per pipeline stage
+constexpr int kStages = 4;
+constexpr int ROWW = BKW + 4;    // padded smem row stride in words (80 B)
+constexpr int kSmemBytes = kStages * (BM + BN) * ROWW * 4;   // 80 KiB
+}  // namespace sad
+
+__device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm("vabsdiff4.u32.u32.u32.add %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+
+__device__ __forceinline__ void cp_async16(uint32_t* smem, const void* gmem) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+// A: input tiles, rows [0, nrows) (already offset by row_begin); B: target
+// tiles, rows [0, S).  kw_split: K words handled by one blockIdx.z slice.
+template <bool kAtomic>
+__global__ void __launch_bounds__(sad::kThreads, 1)
+k_sad(const uint8_t* __restrict__ A, const uint8_t* __restrict__ B, int64_t ldt, int32_t nrows,
+      int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE) {
+  using namespace sad;
+  extern __shared__ __align__(16) uint32_t smem[];
+  uint32_t* sA = smem;                                 // [kStages][BM][ROWW]
+  uint32_t* sB = smem + kStages * BM * ROWW;           // [kStages][BN][ROWW]
+
+  const int tid = threadIdx.x;
+  const int tx = tid & 15, ty = tid >> 4;
+  const int32_t row0 = blockIdx.y * BM, col0 = blockIdx.x * BN;
+  const int64_t kbyte0 = (int64_t)blockIdx.z * kw_split * 4;
+  const int nkb = kw_split / BKW;
+
+  // Loader: per operand and stage, BM rows x 64 B = 512 16-byte chunks; thread
+  // tid copies chunks q = tid and q = tid + 256 (row q >> 2, part q & 3).
+  const uint8_t* srcA[2];
+  const uint8_t* srcB[2];
+  int dst_off[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const int q = tid + h * kThreads;
+    const int r = q >> 2, part = q & 3;
+    int32_t ra = row0 + r; if (ra >= nrows) ra = nrows - 1;   // clamp: loaded, never stored
+    int32_t rb = col0 + r; if (rb >= S) rb = S - 1;
+    srcA[h] = A + (int64_t)ra * ldt + kbyte0 + part * 16;
+    srcB[h] = B + (int64_t)rb * ldt + kbyte0 + part * 16;
+    dst_off[h] = r * ROWW + part * 4;
+  }
+  auto load_stage = [&](int kb, int stage) {
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      cp_async16(sA + stage * BM * ROWW + dst_off[h], srcA[h] + kb * (BKW * 4));
+      cp_async16(sB + stage * BN * ROWW + dst_off[h], srcB[h] + kb * (BKW * 4));
+    }
+  };
+
+  uint32_t acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0u;
+
+#pragma unroll
+  for (int s = 0; s < kStages - 1; ++s) {
+    if (s < nkb) load_stage(s, s);
+    cp_async_commit();
+  }
+
+  for (int kb = 0; kb < nkb; ++kb) {
+    cp_async_wait<kStages - 2>();
+    __syncthreads();   // stage kb landed for all; stage kb-1 fully consumed
+    {
+      const int nk = kb + kStages - 1;
+      if (nk < nkb) load_stage(nk, nk % kStages);
+      cp_async_commit();
+    }
+    const int stage = kb % kStages;
+    const uint32_t* a_base = sA + stage * BM * ROWW + ty * ROWW;
+    const uint32_t* b_base = sB + stage * BN * ROWW + tx * ROWW;
+#pragma unroll
+    for (int kk = 0; kk < BKW; kk += 4) {
+      uint4 a[8], b[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) a[i] = *reinterpret_cast<const uint4*>(a_base + i * 16 * ROWW + kk);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) b[j] = *reinterpret_cast<const uint4*>(b_base + j * 16 * ROWW + kk);
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          uint32_t t = acc[i][j];
+          t = sad4(a[i].x, b[j].x, t);
+          t = sad4(a[i].y, b[j].y, t);
+          t = sad4(a[i].z, b[j].z, t);
+          t = sad4(a[i].w, b[j].w, t);
+          acc[i][j] = t;
+        }
+    }
+  }
+  cp_async_wait<0>();
+
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int32_t row = row0 + ty + 16 * i;
+    if (row >= nrows) continue;
+    int32_t* erow = E + (int64_t)row * ldE;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int32_t col = col0 + tx + 16 * j;
+      if (col >= S) continue;
+      if (kAtomic) atomicAdd(erow + col, (int32_t)acc[i][j]);
+      else erow[col] = (int32_t)acc[i][j];
+    }
+  }
+}
+
+// Host-side split-K choice: minimise waves(tiles * split) * (nkb / split) over
+// the divisors of nkb that leave >= 2 K-chunks per CTA.
+static int choose_split(int64_t tiles, int nkb, int sms) {
+  int best = 1;
+  double best_cost = 1e300;
+  for (int s = 1; s <= nkb; ++s) {
+    if (nkb % s) continue;
+    if (s > 1 && nkb / s < 2) break;
+    const int64_t ctas = tiles * s;
+    const int64_t waves = (ctas + sms - 1) / sms;
+    // small bias against splitting (memset + atomics)
+    const double cost = (double)waves * (nkb / s) * (s > 1 ? 1.03 : 1.0);
+    if (cost < best_cost - 1e-9) { best_cost = cost; best = s; }
+  }
+  return best;
+}
+
+cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
+                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st) {
+  using namespace sad;
+  (void)P;
+  if (nrows <= 0 || S <= 0) return cudaSuccess;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  static std::atomic<uint64_t> attr_done{0};   // one bit per device ordinal
+  if (dev < 64 && !(attr_done.load() & (1ull << dev))) {
+    cudaError_t e = cudaFuncSetAttribute(k_sad<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(k_sad<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_done.fetch_or(1ull << dev);
+  }
+  const int kw = (int)(ldt / 4);
+  const int nkb = kw / BKW;
+  const int64_t gx = (S + BN - 1) / BN, gy = (nrows + BM - 1) / BM;
+  if (gy > 65535) return cudaErrorInvalidValue;
+  const int split = choose_split(gx * gy, nkb, sms);
+  dim3 grid((unsigned)gx, (unsigned)gy, (unsigned)split);
+  if (split > 1) {
+    // split-K accumulates with red.add: zero the [nrows][S] window of E first
+    cudaError_t e = (ldE == S)
+        ? cudaMemsetAsync(E, 0, sizeof(int32_t) * (size_t)nrows * S, st)
+        : cudaMemset2DAsync(E, sizeof(int32_t) * ldE, 0, sizeof(int32_t) * S, nrows, st);
+    if (e != cudaSuccess) return e;
+    k_sad<true><<<grid, kThreads, kSmemBytes, st>>>(A, B, ldt, nrows, S, kw / split, E, ldE);
+  } else {
+    k_sad<false><<<grid, kThreads, kSmemBytes, st>>>(A, B, ldt, nrows, S, kw, E, ldE);
+  }
+  note_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace pm

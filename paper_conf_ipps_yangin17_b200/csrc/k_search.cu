@@ -1,0 +1,358 @@
+// k_search.cu -- Step 3, the parallel approximation (Algorithm 2)
+// and the total error (Eq. 2) for sm_100a.
+//
+// State: r[u] = input tile at target slot u (reading R5) and the maintained
+// diagonal d[u] = E[r[u]][u].  A pair (u, v) of class c, a = r[u], b = r[v],
+// fires iff d[u] + d[v] > E[b][u] + E[a][v] (line 5, strict: reading R6); on a
+// swap r[u] = b, r[v] = a, d[u] = E[b][u], d[v] = E[a][v].  This is line 5's
+// four-entry test with two of the entries carried in d (the oracle evaluates
+// all four every time), so each pair costs two gathers from E.
+//
+// Methods (pm_ls_method_t):
+//   CLASS  -- the paper's structure: one kernel per colour class, the
+//             n-1 class launches of a round captured once into a CUDA graph
+//             whose while-node repeats rounds on the device until a round
+//             has no swap (no host round trip per round).
+//   CTA    -- one CTA runs every round: r and d in shared memory, a
+//             __syncthreads() between classes instead of a kernel boundary.
+#include <cuda_runtime.h>
+
+#include <map>
+#include <mutex>
+#include <tuple>
+
+#include "pm_internal.cuh"
+
+namespace pm {
+
+// Device-resident parameters of one search (fixed address per cached graph).
+struct LsParams {
+  const int32_t* E;
+  int64_t ldE;
+  int32_t* r;
+  int32_t* d;          // maintained diagonal, int32 [S] (CLASS method scratch)
+  int32_t* seen;       // permutation check, int32 [S]
+  int32_t S;
+  int32_t max_rounds;
+  int32_t max_log;
+  int32_t pad;
+  unsigned long long round_swaps;
+  LsResult* out;
+  int64_t* per_round;
+};
+
+// ------------------------------------------------------------- CLASS -----
+// Parameters travel as a kernel argument (no pageable H2D copy, no host sync).
+__global__ void k_ls_set_params(LsParams* dst, LsParams src) { *dst = src; }
+
+__global__ void k_ls_check_init(LsParams* p) {
+  const int32_t S = p->S;
+  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x) {
+    const int32_t t = p->r[u];
+    if (t < 0 || t >= S) {
+      p->out->status = PM_ERR_NOT_PERMUTATION;
+      continue;
+    }
+    atomicAdd(p->seen + t, 1);
+    p->d[u] = p->E[(int64_t)t * p->ldE + u];
+  }
+}
+
+__global__ void k_ls_check_seen(LsParams* p) {
+  const int32_t S = p->S;
+  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x)
+    if (p->seen[u] != 1) p->out->status = PM_ERR_NOT_PERMUTATION;
+}
+
+// One colour class P_{c+1}: every pair concurrently (Alg. 2 line 4).
+__global__ void __launch_bounds__(256) k_ls_class(const LsParams* __restrict__ p, int32_t c) {
+  if (p->out->status != PM_OK) return;
+  const Classes cl(p->S);
+  const int32_t k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= cl.npairs) return;
+  int32_t u, v;
+  cl.pair(c, k, u, v);
+  int32_t* r = p->r;
+  int32_t* d = p->d;
+  const int32_t* E = p->E;
+  const int64_t ld = p->ldE;
+  const int32_t a = r[u], b = r[v];
+  const int32_t e_bu = __ldg(E + (int64_t)b * ld + u);
+  const int32_t e_av = __ldg(E + (int64_t)a * ld + v);
+  const int32_t du = d[u], dv = d[v];
+  if ((int64_t)du + dv > (int64_t)e_bu + e_av) {
+    r[u] = b; r[v] = a;
+    d[u] = e_bu; d[v] = e_av;
+    atomicAdd(const_cast<unsigned long long*>(&p->round_swaps), 1ull);
+  }
+}
+
+// Alg. 2 line 11 (+ the max_rounds cap): decide whether the while-node loops.
+__global__ void k_ls_round_end(LsParams* p, cudaGraphConditionalHandle h) {
+  LsResult* o = p->out;
+  unsigned cont = 0;
+  if (o->status == PM_OK) {
+    const int64_t sw = (int64_t)p->round_swaps;
+    p->round_swaps = 0;
+    if (o->rounds < p->max_log) p->per_round[o->rounds] = sw;
+    o->rounds += 1;
+    o->swaps += sw;
+    if (sw > 0) {
+      if (p->max_rounds > 0 && o->rounds >= p->max_rounds) o->status = PM_ERR_NOT_CONVERGED;
+      else cont = 1;
+    }
+  }
+  cudaGraphSetConditional(h, cont);
+}
+
+struct ClassGraph {
+  LsParams* dparams = nullptr;
+  cudaGraphExec_t exec = nullptr;
+};
+
+static std::mutex g_graph_mu;
+static std::map<std::tuple<int, int32_t, cudaStream_t>, ClassGraph> g_graphs;
+
+static cudaError_t build_class_graph(int32_t S, cudaStream_t st, ClassGraph& out) {
+  const Classes cl(S);
+  cudaError_t e = cudaMalloc(&out.dparams, sizeof(LsParams));
+  if (e != cudaSuccess) return e;
+  cudaGraph_t g = nullptr;
+  if ((e = cudaGraphCreate(&g, 0)) != cudaSuccess) return e;
+  cudaGraphConditionalHandle h;
+  if ((e = cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault)) != cudaSuccess) return e;
+  cudaGraphNodeParams cp = {};
+  cp.type = cudaGraphNodeTypeConditional;
+  cp.conditional.handle = h;
+  cp.conditional.type = cudaGraphCondTypeWhile;
+  cp.conditional.size = 1;
+  cudaGraphNode_t node;
+  if ((e = cudaGraphAddNode(&node, g, nullptr, 0, &cp)) != cudaSuccess) return e;
+  cudaGraph_t body = cp.conditional.phGraph_out[0];
+  // Populate the loop body by capturing one round onto a private stream.
+  cudaStream_t cs;
+  if ((e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking)) != cudaSuccess) return e;
+  if ((e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed)) != cudaSuccess)
+    return e;
+  const int threads = 256;
+  const int blocks = (cl.npairs + threads - 1) / threads;
+  for (int32_t c = 0; c < cl.ncls; ++c) k_ls_class<<<blocks > 0 ? blocks : 1, threads, 0, cs>>>(out.dparams, c);
+  k_ls_round_end<<<1, 1, 0, cs>>>(out.dparams, h);
+  cudaGraph_t captured = body;
+  e = cudaStreamEndCapture(cs, &captured);
+  cudaStreamDestroy(cs);
+  if (e != cudaSuccess) return e;
+  e = cudaGraphInstantiate(&out.exec, g, 0);
+  cudaGraphDestroy(g);
+  (void)st;
+  return e;
+}
+
+static pm_status_t run_class(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                             LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
+  int dev = 0;
+  PM_CUDA_TRY(cudaGetDevice(&dev));
+  ClassGraph cg;
+  {
+    std::lock_guard<std::mutex> lk(g_graph_mu);
+    auto key = std::make_tuple(dev, S, st);
+    auto it = g_graphs.find(key);
+    if (it == g_graphs.end()) {
+      ClassGraph ng;
+      PM_CUDA_TRY(build_class_graph(S, st, ng));
+      it = g_graphs.emplace(key, ng).first;
+    }
+    cg = it->second;
+  }
+  int32_t* scratch = nullptr;   // d [S] + seen [S]
+  PM_CUDA_TRY(cudaMallocAsync(&scratch, sizeof(int32_t) * 2 * (size_t)(S > 0 ? S : 1), st));
+  PM_CUDA_TRY(cudaMemsetAsync(scratch + S, 0, sizeof(int32_t) * (size_t)S, st));
+  LsParams hp = {};
+  hp.E = E; hp.ldE = ldE; hp.r = perm; hp.d = scratch; hp.seen = scratch + S;
+  hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
+  hp.round_swaps = 0; hp.out = dev_out; hp.per_round = dev_per_round;
+  k_ls_set_params<<<1, 1, 0, st>>>(cg.dparams, hp);
+  const int blocks = (S + 255) / 256 > 0 ? (S + 255) / 256 : 1;
+  k_ls_check_init<<<blocks, 256, 0, st>>>(cg.dparams);
+  k_ls_check_seen<<<blocks, 256, 0, st>>>(cg.dparams);
+  note_launch(3);
+  PM_CUDA_TRY(cudaGetLastError());
+  PM_CUDA_TRY(cudaGraphLaunch(cg.exec, st));
+  // the graph's launches (rounds * (ncls + 1)) are counted by the caller once
+  // it has read `rounds` back
+  PM_CUDA_TRY(cudaFreeAsync(scratch, st));
+  return PM_OK;
+}
+
+// --------------------------------------------------------------- CTA -----
+// One CTA, kThreads threads, runs Algorithm 2 to convergence.  Dynamic smem:
+// r [S] and d [S] (int32) + a small reduction area.
+constexpr int kCtaThreads = 1024;
+
+__device__ __forceinline__ int block_sum(int v, int* s_red) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  __syncthreads();
+  if (l == 0) s_red[w] = v;
+  __syncthreads();
+  int t = 0;
+  if (threadIdx.x < 32) {
+    t = (threadIdx.x < (blockDim.x >> 5)) ? s_red[threadIdx.x] : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+    if (threadIdx.x == 0) s_red[32] = t;
+  }
+  __syncthreads();
+  return s_red[32];
+}
+
+__global__ void __launch_bounds__(kCtaThreads, 1)
+k_ls_cta(const int32_t* __restrict__ E, int64_t ld, int32_t S, int32_t* __restrict__ perm,
+         int32_t max_rounds, LsResult* out, int64_t* per_round, int32_t max_log) {
+  extern __shared__ int32_t sm[];
+  int32_t* s_r = sm;
+  int32_t* s_d = sm + S;
+  int* s_red = sm + 2 * S;        // 33 ints
+  const Classes cl(S);
+  const int T = blockDim.x;
+
+  // Permutation check (r is a bijection), then d[u] = E[r[u]][u].
+  for (int32_t x = threadIdx.x; x < S; x += T) s_d[x] = 0;
+  __syncthreads();
+  int bad = 0;
+  for (int32_t u = threadIdx.x; u < S; u += T) {
+    const int32_t t = perm[u];
+    s_r[u] = t;
+    if (t < 0 || t >= S) bad = 1;
+    else atomicAdd(&s_d[t], 1);
+  }
+  __syncthreads();
+  for (int32_t x = threadIdx.x; x < S; x += T)
+    if (s_d[x] != 1) bad = 1;
+  if (__syncthreads_or(bad)) {
+    if (threadIdx.x == 0) { out->status = PM_ERR_NOT_PERMUTATION; out->rounds = 0; out->swaps = 0; }
+    return;
+  }
+  for (int32_t u = threadIdx.x; u < S; u += T) s_d[u] = __ldg(E + (int64_t)s_r[u] * ld + u);
+  __syncthreads();
+
+  int32_t rounds = 0;
+  int64_t total = 0;
+  int status = PM_OK;
+  for (;;) {
+    int mysw = 0;
+    for (int32_t c = 0; c < cl.ncls; ++c) {
+      for (int32_t k = threadIdx.x; k < cl.npairs; k += T) {
+        int32_t u, v;
+        cl.pair(c, k, u, v);
+        const int32_t a = s_r[u], b = s_r[v];
+        const int32_t e_bu = __ldg(E + (int64_t)b * ld + u);
+        const int32_t e_av = __ldg(E + (int64_t)a * ld + v);
+        const int32_t du = s_d[u], dv = s_d[v];
+        if ((int64_t)du + dv > (int64_t)e_bu + e_av) {
+          s_r[u] = b; s_r[v] = a;
+          s_d[u] = e_bu; s_d[v] = e_av;
+          ++mysw;
+        }
+      }
+      __syncthreads();
+    }
+    const int sw = block_sum(mysw, s_red);
+    if (threadIdx.x == 0 && rounds < max_log) per_round[rounds] = sw;
+    rounds += 1;
+    total += sw;
+    if (sw == 0) break;
+    if (max_rounds > 0 && rounds >= max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
+  }
+  for (int32_t u = threadIdx.x; u < S; u += T) perm[u] = s_r[u];
+  if (threadIdx.x == 0) { out->status = status; out->rounds = rounds; out->swaps = total; }
+}
+
+static int32_t cta_smem_bytes(int32_t S) { return (int32_t)(sizeof(int32_t) * (2 * (size_t)S + 40)); }
+
+int32_t ls_cta_max_S() {
+  int dev = 0, optin = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  if (cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) return 0;
+  return (int32_t)((optin / 4 - 40) / 2);
+}
+
+static pm_status_t run_cta(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                           LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
+  const int32_t smem = cta_smem_bytes(S);
+  PM_CUDA_TRY(cudaFuncSetAttribute(k_ls_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  int threads = kCtaThreads;
+  while (threads > 64 && threads / 2 >= (S / 2)) threads /= 2;   // small S: fewer idle warps
+  k_ls_cta<<<1, threads, smem, st>>>(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log);
+  note_launch();
+  PM_CUDA_TRY(cudaGetLastError());
+  return PM_OK;
+}
+
+pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                             int32_t method, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
+                             cudaStream_t st, int32_t* used_method) {
+  const int32_t cta_max = ls_cta_max_S();
+  if (method == PM_LS_AUTO) method = (S <= cta_max) ? PM_LS_CTA : PM_LS_CLASS;
+  if (used_method) *used_method = method;
+  switch (method) {
+    case PM_LS_CLASS:
+      return run_class(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+    case PM_LS_CTA:
+      if (S > cta_max) return PM_ERR_UNSUPPORTED;
+      return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+    default:
+      return PM_ERR_UNSUPPORTED;
+  }
+}
+
+// ------------------------------------------------------------ Eq. (2) ----
+__global__ void __launch_bounds__(256) k_cost(const int32_t* __restrict__ E, int64_t ld, int32_t S,
+                                              const int32_t* __restrict__ perm,
+                                              unsigned long long* __restrict__ cost) {
+  long long s = 0;
+  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x)
+    s += __ldg(E + (int64_t)__ldg(perm + u) * ld + u);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  __shared__ long long red[8];
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    long long t = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+    atomicAdd(cost, (unsigned long long)t);
+  }
+}
+
+cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm, int64_t* d_cost,
+                        cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(d_cost, 0, sizeof(int64_t), st);
+  if (e != cudaSuccess) return e;
+  int blocks = (S + 255) / 256;
+  if (blocks < 1) blocks = 1;
+  if (blocks > 148) blocks = 148;
+  k_cost<<<blocks, 256, 0, st>>>(E, ldE, S, perm, reinterpret_cast<unsigned long long*>(d_cost));
+  note_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace pm
+
+namespace pm {
+int32_t ls_class_launches_per_round(int32_t S) { return Classes(S).ncls + 1; }
+
+// r := identity (Alg. 1/2 start from the input image as given, reading R7).
+__global__ void k_iota(int32_t* perm, int32_t S) {
+  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x) perm[u] = u;
+}
+cudaError_t launch_iota(int32_t* perm, int32_t S, cudaStream_t st) {
+  int blocks = (S + 255) / 256;
+  if (blocks < 1) blocks = 1;
+  if (blocks > 1184) blocks = 1184;
+  k_iota<<<blocks, 256, 0, st>>>(perm, S);
+  note_launch();
+  return cudaGetLastError();
+}
+}  // namespace pm

@@ -1,0 +1,283 @@
+// pm_abi.cu -- the extern "C" entry points of libpm.so (include/pm.h):
+// argument validation, scratch management and the calls into the kernels of
+// k_sad.cu / k_search.cu.  No compute happens here; there is no CPU fallback.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "pm_internal.cuh"
+
+namespace pm {
+std::atomic<int64_t> g_launches{0};
+}  // namespace pm
+
+using namespace pm;
+
+namespace {
+
+constexpr int32_t kMaxLog = 1024;   // per-round swap log kept on the device
+
+bool valid_image_args(int32_t N, int32_t M, int32_t C) {
+  if (N <= 0 || M <= 0 || C <= 0) return false;
+  if (N % M != 0) return false;                        // P:57, S = (N/M)^2
+  const int64_t P = (int64_t)M * M * C;
+  if (P * 255 > INT32_MAX) return false;               // reading R11: int32 E
+  const int64_t g = N / M;
+  if (g * g > INT32_MAX / 2) return false;
+  return true;
+}
+
+struct DevBuf {
+  void* p = nullptr;
+  cudaStream_t st = nullptr;
+  ~DevBuf() { if (p) cudaFreeAsync(p, st); }
+};
+
+bool valid_ls_args(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int32_t max_rounds,
+                   int32_t method) {
+  if (!d_E || !d_perm || S < 1 || ld_E < S || max_rounds < 0) return false;
+  return method >= PM_LS_AUTO && method <= PM_LS_WINDOW;
+}
+
+// Synchronous local search: scratch, launch, read back.
+pm_status_t local_search_impl(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                              int32_t max_rounds, int32_t method, int32_t* h_rounds, int64_t* h_swaps,
+                              int64_t* h_per_round, int32_t len, cudaStream_t st) {
+  if (!valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method)) return PM_ERR_INVALID;
+  DevBuf buf;
+  buf.st = st;
+  const size_t bytes = sizeof(LsResult) + sizeof(int64_t) * kMaxLog;
+  PM_CUDA_TRY(cudaMallocAsync(&buf.p, bytes, st));
+  LsResult* dres = reinterpret_cast<LsResult*>(buf.p);
+  int64_t* dlog = reinterpret_cast<int64_t*>(reinterpret_cast<char*>(buf.p) + sizeof(LsResult));
+  PM_CUDA_TRY(cudaMemsetAsync(buf.p, 0, bytes, st));
+  int32_t used = method;
+  pm_status_t s = run_local_search(d_E, ld_E, S, d_perm, max_rounds, method, dres, dlog, kMaxLog, st, &used);
+  if (s != PM_OK) return s;
+  LsResult hres;
+  std::vector<int64_t> hlog;
+  PM_CUDA_TRY(cudaMemcpyAsync(&hres, dres, sizeof(hres), cudaMemcpyDeviceToHost, st));
+  if (h_per_round && len > 0) {
+    hlog.resize(std::min(len, kMaxLog));
+    PM_CUDA_TRY(cudaMemcpyAsync(hlog.data(), dlog, sizeof(int64_t) * hlog.size(), cudaMemcpyDeviceToHost, st));
+  }
+  PM_CUDA_TRY(cudaStreamSynchronize(st));
+  if (used == PM_LS_CLASS) note_launch(hres.rounds * ls_class_launches_per_round(S));
+  if (h_rounds) *h_rounds = (int32_t)hres.rounds;
+  if (h_swaps) *h_swaps = hres.swaps;
+  if (h_per_round && len > 0) {
+    const int32_t n = (int32_t)std::min<int64_t>(hres.rounds, (int64_t)hlog.size());
+    for (int32_t i = 0; i < n; ++i) h_per_round[i] = hlog[i];
+  }
+  return (pm_status_t)hres.status;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* pm_status_string(pm_status_t s) {
+  switch (s) {
+    case PM_OK: return "PM_OK";
+    case PM_ERR_INVALID: return "PM_ERR_INVALID: invalid argument";
+    case PM_ERR_CUDA: return "PM_ERR_CUDA: CUDA runtime error";
+    case PM_ERR_NOT_CONVERGED: return "PM_ERR_NOT_CONVERGED: max_rounds reached before a zero-swap round";
+    case PM_ERR_UNSUPPORTED: return "PM_ERR_UNSUPPORTED: not supported by this build/device";
+    case PM_ERR_NOT_PERMUTATION: return "PM_ERR_NOT_PERMUTATION: perm is not a bijection of [0, S)";
+  }
+  return "PM_ERR_?: unknown status";
+}
+
+int64_t pm_tile_stride(int32_t M, int32_t C) {
+  if (M <= 0 || C <= 0) return 0;
+  const int64_t P = (int64_t)M * M * C;
+  return (P + 63) / 64 * 64;
+}
+
+pm_status_t pm_pack_tiles(const uint8_t* d_img, int32_t N, int32_t M, int32_t C, uint8_t* d_tiles,
+                          int64_t ld_tiles, pm_stream_t stream) {
+  if (!d_img || !d_tiles || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  if (ld_tiles < (int64_t)M * M * C || ld_tiles % 16 != 0) return PM_ERR_INVALID;
+  const int32_t g = N / M;
+  PM_CUDA_TRY(launch_pack(d_img, N, M, C, d_tiles, ld_tiles, 0, g * g, (cudaStream_t)stream));
+  return PM_OK;
+}
+
+pm_status_t pm_error_matrix_tiles(const uint8_t* d_input_tiles, const uint8_t* d_target_tiles,
+                                  int64_t ld_tiles, int32_t S, int32_t P, int32_t row_begin, int32_t row_end,
+                                  int32_t* d_E, int64_t ld_E, pm_stream_t stream) {
+  if (!d_input_tiles || !d_target_tiles || !d_E) return PM_ERR_INVALID;
+  if (S < 1 || P < 1 || (int64_t)P * 255 > INT32_MAX) return PM_ERR_INVALID;
+  if (ld_tiles < P || ld_tiles % 64 != 0) return PM_ERR_INVALID;
+  if (row_begin < 0 || row_end > S || row_begin > row_end || ld_E < S) return PM_ERR_INVALID;
+  PM_CUDA_TRY(launch_sad(d_input_tiles + (int64_t)row_begin * ld_tiles, d_target_tiles, ld_tiles,
+                         row_end - row_begin, S, P, d_E, ld_E, (cudaStream_t)stream));
+  return PM_OK;
+}
+
+pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M, int32_t C,
+                            int32_t row_begin, int32_t row_end, int32_t* d_E, int64_t ld_E,
+                            pm_stream_t stream) {
+  if (!d_input || !d_target || !d_E || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  const int32_t g = N / M;
+  const int32_t S = g * g;
+  if (row_begin < 0 || row_end > S || row_begin > row_end || ld_E < S) return PM_ERR_INVALID;
+  if (row_begin == row_end) return PM_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t ldt = pm_tile_stride(M, C);
+  const int32_t nrows = row_end - row_begin;
+  DevBuf buf;
+  buf.st = st;
+  PM_CUDA_TRY(cudaMallocAsync(&buf.p, (size_t)ldt * ((size_t)nrows + S), st));
+  uint8_t* tI = reinterpret_cast<uint8_t*>(buf.p);
+  uint8_t* tT = tI + (size_t)ldt * nrows;
+  PM_CUDA_TRY(launch_pack(d_input, N, M, C, tI, ldt, row_begin, row_end, st));
+  PM_CUDA_TRY(launch_pack(d_target, N, M, C, tT, ldt, 0, S, st));
+  PM_CUDA_TRY(launch_sad(tI, tT, ldt, nrows, S, M * M * C, d_E, ld_E, st));
+  return PM_OK;
+}
+
+int32_t pm_num_colors(int32_t S) { return Classes(S).ncls; }
+
+pm_status_t pm_edge_coloring(int32_t S, int32_t class_begin, int32_t class_end, int32_t* h_pairs) {
+  const Classes cl(S);
+  if (S < 2 || !h_pairs || class_begin < 0 || class_end > cl.ncls || class_begin > class_end)
+    return PM_ERR_INVALID;
+  const int32_t per = S / 2;
+  std::vector<std::pair<int32_t, int32_t>> grp;
+  for (int32_t c = class_begin; c < class_end; ++c) {
+    grp.clear();
+    for (int32_t k = 0; k < cl.npairs; ++k) {
+      int32_t u, v;
+      cl.pair(c, k, u, v);
+      grp.emplace_back(std::min(u, v), std::max(u, v));
+    }
+    std::sort(grp.begin(), grp.end());   // the paper lists pairs by smaller index
+    int32_t* out = h_pairs + (int64_t)(c - class_begin) * per * 2;
+    int32_t k = 0;
+    for (; k < (int32_t)grp.size(); ++k) { out[2 * k] = grp[k].first; out[2 * k + 1] = grp[k].second; }
+    for (; k < per; ++k) { out[2 * k] = -1; out[2 * k + 1] = -1; }
+  }
+  return PM_OK;
+}
+
+pm_status_t pm_local_search(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm, int32_t max_rounds,
+                            int32_t* h_rounds, int64_t* h_swaps, pm_stream_t stream) {
+  return local_search_impl(d_E, ld_E, S, d_perm, max_rounds, PM_LS_AUTO, h_rounds, h_swaps, nullptr, 0,
+                           (cudaStream_t)stream);
+}
+
+pm_status_t pm_local_search_ex(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm, int32_t max_rounds,
+                               int32_t method, int32_t* h_rounds, int64_t* h_swaps, int64_t* h_swaps_per_round,
+                               int32_t len, pm_stream_t stream) {
+  return local_search_impl(d_E, ld_E, S, d_perm, max_rounds, method, h_rounds, h_swaps, h_swaps_per_round, len,
+                           (cudaStream_t)stream);
+}
+
+pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                  int32_t max_rounds, int32_t method, int64_t* d_result, pm_stream_t stream) {
+  if (!d_result || !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method)) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
+  int32_t used = method;
+  return run_local_search(d_E, ld_E, S, d_perm, max_rounds, method, reinterpret_cast<LsResult*>(d_result),
+                          nullptr, 0, st, &used);
+}
+
+int32_t pm_ls_cta_max_S(void) { return ls_cta_max_S(); }
+
+pm_status_t pm_cost_async(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int64_t* d_cost,
+                          pm_stream_t stream) {
+  if (!d_E || !d_perm || !d_cost || S < 1 || ld_E < S) return PM_ERR_INVALID;
+  PM_CUDA_TRY(launch_cost(d_E, ld_E, S, d_perm, d_cost, (cudaStream_t)stream));
+  return PM_OK;
+}
+
+pm_status_t pm_cost(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int64_t* h_cost,
+                    pm_stream_t stream) {
+  if (!h_cost) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  DevBuf buf;
+  buf.st = st;
+  PM_CUDA_TRY(cudaMallocAsync(&buf.p, sizeof(int64_t), st));
+  pm_status_t s = pm_cost_async(d_E, ld_E, S, d_perm, reinterpret_cast<int64_t*>(buf.p), stream);
+  if (s != PM_OK) return s;
+  PM_CUDA_TRY(cudaMemcpyAsync(h_cost, buf.p, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+  PM_CUDA_TRY(cudaStreamSynchronize(st));
+  return PM_OK;
+}
+
+pm_status_t pm_init_identity(int32_t* d_perm, int32_t S, pm_stream_t stream) {
+  if (!d_perm || S < 1) return PM_ERR_INVALID;
+  PM_CUDA_TRY(launch_iota(d_perm, S, (cudaStream_t)stream));
+  return PM_OK;
+}
+
+pm_status_t pm_photomosaic_async(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M, int32_t C,
+                                 int32_t* d_E, int64_t ld_E, int32_t* d_perm, int32_t method, int64_t* d_result,
+                                 pm_stream_t stream) {
+  if (!d_input || !d_target || !d_E || !d_perm || !d_result || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  if (method < PM_LS_AUTO || method > PM_LS_WINDOW) return PM_ERR_INVALID;
+  const int32_t g = N / M;
+  const int32_t S = g * g;
+  if (ld_E < S) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  pm_status_t s = pm_error_matrix(d_input, d_target, N, M, C, 0, S, d_E, ld_E, stream);   // Steps 1-2
+  if (s != PM_OK) return s;
+  PM_CUDA_TRY(launch_iota(d_perm, S, st));                                                // r = identity
+  s = pm_local_search_async(d_E, ld_E, S, d_perm, 0, method, d_result, stream);           // Alg. 2
+  if (s != PM_OK) return s;
+  PM_CUDA_TRY(launch_cost(d_E, ld_E, S, d_perm, d_result + 3, st));                       // Eq. (2)
+  return PM_OK;
+}
+
+pm_status_t pm_photomosaic(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M, int32_t C,
+                           int32_t* d_E, int64_t ld_E, int32_t* d_perm, int32_t method, int32_t* h_rounds,
+                           int64_t* h_swaps, int64_t* h_cost, pm_stream_t stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  DevBuf buf;   // {status, rounds, swaps, cost}
+  buf.st = st;
+  if (!d_input || !d_target || !d_E || !d_perm || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  PM_CUDA_TRY(cudaMallocAsync(&buf.p, 4 * sizeof(int64_t), st));
+  pm_status_t s = pm_photomosaic_async(d_input, d_target, N, M, C, d_E, ld_E, d_perm, method,
+                                       reinterpret_cast<int64_t*>(buf.p), stream);
+  if (s != PM_OK) return s;
+  int64_t h[4];
+  PM_CUDA_TRY(cudaMemcpyAsync(h, buf.p, sizeof(h), cudaMemcpyDeviceToHost, st));
+  PM_CUDA_TRY(cudaStreamSynchronize(st));
+  if (h_rounds) *h_rounds = (int32_t)h[1];
+  if (h_swaps) *h_swaps = h[2];
+  if (h_cost) *h_cost = h[3];
+  return (pm_status_t)h[0];
+}
+
+pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target, int32_t N, int32_t M, int32_t C,
+                                int32_t method, int32_t* h_perm, int32_t* h_rounds, int64_t* h_swaps,
+                                int64_t* h_cost, pm_stream_t stream) {
+  if (!h_input || !h_target || !h_perm || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int32_t g = N / M;
+  const int64_t S = (int64_t)g * g;
+  const size_t img = (size_t)N * N * C;
+  const size_t bytes = 2 * img + sizeof(int32_t) * (size_t)S * (size_t)S + sizeof(int32_t) * (size_t)S + 64;
+  DevBuf buf;
+  buf.st = st;
+  PM_CUDA_TRY(cudaMallocAsync(&buf.p, bytes, st));
+  char* base = reinterpret_cast<char*>(buf.p);
+  int32_t* dE = reinterpret_cast<int32_t*>(base);
+  int32_t* dperm = dE + S * S;
+  uint8_t* dI = reinterpret_cast<uint8_t*>(dperm + S);
+  uint8_t* dT = dI + img;
+  PM_CUDA_TRY(cudaMemcpyAsync(dI, h_input, img, cudaMemcpyHostToDevice, st));
+  PM_CUDA_TRY(cudaMemcpyAsync(dT, h_target, img, cudaMemcpyHostToDevice, st));
+  pm_status_t s = pm_photomosaic(dI, dT, N, M, C, dE, S, dperm, method, h_rounds, h_swaps, h_cost, stream);
+  if (s != PM_OK) return s;
+  PM_CUDA_TRY(cudaMemcpyAsync(h_perm, dperm, sizeof(int32_t) * (size_t)S, cudaMemcpyDeviceToHost, st));
+  PM_CUDA_TRY(cudaStreamSynchronize(st));
+  return PM_OK;
+}
+
+int64_t pm_launch_count(void) { return g_launches.load(); }
+
+}  // extern "C"

@@ -1,0 +1,97 @@
+// pm_internal.cuh -- shared internals of libpm.so (CUDA path only; the CPU
+// oracle under oracle/ shares nothing with this file).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <atomic>
+
+#include "../../include/pm.h"
+
+namespace pm {
+
+// ----------------------------------------------------------------------------
+// Launch accounting (pm_launch_count): every kernel launch in this library
+// goes through note_launch().
+extern std::atomic<int64_t> g_launches;
+inline void note_launch(int64_t n = 1) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+#define PM_CUDA_TRY(expr)                         \
+  do {                                            \
+    cudaError_t _e = (expr);                      \
+    if (_e != cudaSuccess) return PM_ERR_CUDA;    \
+  } while (0)
+
+// ----------------------------------------------------------------------------
+// Colour classes of K_S (Theorem 1; groups P:152-203), generated on the
+// fly.  0-indexed slots, class c in [0, ncls).  Reading R7: with m = S-1 (S
+// even) or m = S (S odd), class c pairs slots whose sum is 2c+1 (mod m); its
+// fixed point u0 = (c + (m+1)/2) mod m (the solution of 2u0 == 2c+1) is joined
+// to slot S-1 when S is even and idles when S is odd.  Enumerated here as
+// pair k:  k == 0 -> (u0, S-1) [even S];  k >= 1 -> (u0+k, u0-k) mod m.
+struct Classes {
+  int32_t S, m, half, ncls, npairs;  // half = (m+1)/2
+  __host__ __device__ explicit Classes(int32_t S_) : S(S_) {
+    m = (S % 2 == 0) ? S - 1 : S;
+    half = (m + 1) / 2;
+    ncls = (S < 2) ? 0 : m;
+    npairs = S / 2;
+  }
+  __host__ __device__ __forceinline__ int32_t fixed_point(int32_t c) const {
+    int32_t u0 = c + half;
+    return u0 >= m ? u0 - m : u0;
+  }
+  // Pair k in [0, npairs) of class c as (u, v).  (Odd S: the fixed point idles
+  // and is not enumerated.)
+  __host__ __device__ __forceinline__ void pair(int32_t c, int32_t k, int32_t& u, int32_t& v) const {
+    int32_t u0 = fixed_point(c);
+    if (S % 2 == 0) {
+      if (k == 0) { u = u0; v = S - 1; return; }
+    } else {
+      k += 1;  // odd S: pairs k = 1 .. (S-1)/2
+    }
+    int32_t a = u0 + k; if (a >= m) a -= m;
+    int32_t b = u0 - k; if (b < 0) b += m;
+    u = a; v = b;
+  }
+  // Partner of slot x in class c (x itself if it idles: odd S fixed point).
+  __host__ __device__ __forceinline__ int32_t partner(int32_t c, int32_t x) const {
+    int32_t u0 = fixed_point(c);
+    if (S % 2 == 0) {
+      if (x == S - 1) return u0;
+      if (x == u0) return S - 1;
+    } else if (x == u0) {
+      return x;
+    }
+    int32_t p = 2 * c + 1 - x;  // in (-m, 2m)
+    p %= m; if (p < 0) p += m;
+    return p;
+  }
+};
+
+// ----------------------------------------------------------------------------
+// Internal launchers (defined in k_sad.cu / k_search.cu).
+cudaError_t launch_pack(const uint8_t* img, int32_t N, int32_t M, int32_t C, uint8_t* tiles,
+                        int64_t ld_tiles, int32_t tile_begin, int32_t tile_end, cudaStream_t st);
+cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
+                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st);
+
+// Device-side result of one search; layout = the int64 [3] of
+// pm_local_search_async's d_result: {status, rounds, swaps}.
+struct LsResult {
+  int64_t status;  // pm_status_t
+  int64_t rounds;
+  int64_t swaps;
+};
+cudaError_t launch_iota(int32_t* perm, int32_t S, cudaStream_t st);
+int32_t ls_cta_max_S();
+// Runs the whole search; writes device results (LsResult + per-round swaps)
+// into dev_out (LsResult) and dev_per_round (int64 [max_log]).
+pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm,
+                             int32_t max_rounds, int32_t method, LsResult* dev_out,
+                             int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                             int32_t* used_method);
+int32_t ls_class_launches_per_round(int32_t S);
+cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm,
+                        int64_t* d_cost, cudaStream_t st);
+
+}  // namespace pm

@@ -1,0 +1,88 @@
+"""CPU-side checks of the C-ABI boundary (no GPU needed, no compute calls):
+libpm.so loads, exports every function include/pm.h declares, and its
+host-only entry points (pm_num_colors, pm_edge_coloring, pm_tile_stride,
+pm_status_string) behave -- the edge groups checked against the paper's
+printed K_16 table and against the oracle's colouring."""
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "pm.h")
+
+
+def _declared_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(pm_[A-Za-z0-9_]+)\s*\(", src)))
+
+
+@pytest.fixture(scope="module")
+def pm():
+    from paper_conf_ipps_yangin17_b200 import pm as _pm
+    if not os.path.exists(_pm.LIB_PATH):
+        import __graft_entry__
+        __graft_entry__.build()
+    return _pm
+
+
+def test_header_declares_the_boundary():
+    names = _declared_functions()
+    for required in ("pm_error_matrix", "pm_edge_coloring", "pm_local_search", "pm_cost"):
+        assert required in names
+
+
+def test_library_exports_every_declared_symbol(pm):
+    L = pm.lib()
+    missing = [n for n in _declared_functions() if not hasattr(L, n)]
+    assert not missing, f"declared in pm.h but not exported: {missing}"
+    out = subprocess.run(["nm", "-D", "--defined-only", pm.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (pm_[A-Za-z0-9_]+)$", out, flags=re.M))
+    assert set(_declared_functions()) <= exported
+    # the python binding covers the whole ABI
+    assert {n for n, _, _ in pm._SIGS} == set(_declared_functions())
+
+
+def test_library_is_sm100a(pm):
+    out = subprocess.run(["cuobjdump", "--list-elf", pm.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_status_strings(pm):
+    for s in range(6):
+        assert pm.status_string(s).startswith("PM_")
+
+
+def test_tile_stride(pm):
+    assert pm.tile_stride(16, 3) == 768
+    assert pm.tile_stride(8, 3) == 192
+    assert pm.tile_stride(5, 1) == 64
+    assert pm.tile_stride(0, 3) == 0
+
+
+def test_edge_coloring_matches_printed_k16(pm, golden_dir):
+    from tests.test_oracle_coloring import _read_golden
+    gold = _read_golden(os.path.join(golden_dir, "k16_groups.txt"))
+    got = pm.edge_coloring(16)
+    assert pm.num_colors(16) == 15 and got.shape == (15, 8, 2)
+    for i in range(1, 16):
+        assert [tuple(map(int, p)) for p in got[i - 1]] == gold[i], f"P_{i}"
+
+
+@pytest.mark.parametrize("S", [2, 3, 4, 5, 16, 17, 64, 255, 256, 1024])
+def test_edge_coloring_matches_oracle(pm, S):
+    import oracle
+    assert pm.num_colors(S) == oracle.num_colors(S)
+    assert (pm.edge_coloring(S) == oracle.edge_coloring(S)).all()
+
+
+def test_edge_coloring_rejects_bad_ranges(pm):
+    out = np.zeros(16, dtype=np.int32)
+    assert pm.lib().pm_edge_coloring(1, 0, 0, out.ctypes.data) == pm.PM_ERR_INVALID
+    assert pm.lib().pm_edge_coloring(16, 3, 2, out.ctypes.data) == pm.PM_ERR_INVALID
+    assert pm.lib().pm_edge_coloring(16, 0, 16, out.ctypes.data) == pm.PM_ERR_INVALID
+    part = pm.edge_coloring(16, 4, 6)
+    assert (part == pm.edge_coloring(16)[4:6]).all()

@@ -1,0 +1,309 @@
+"""GPU parity: the CUDA path (through the C-ABI, paper_conf_ipps_yangin17_b200.pm)
+against the CPU oracle (oracle/), element by element, on the same seeded
+synthetic inputs.  All results are integers, so the bar is bit-exact:
+E (Eq. 1), the final rearrangement r, rounds, swaps (per round) and the total
+error (Eq. 2).  Full-size configs 4-5 (BASELINE.json) are checked on sampled
+E entries the oracle computes one by one, and the local search there via its
+closed-form special case (transposition) and properties that hold at any
+size (bijection, 2-swap local optimality, cost identity)."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
+
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+DEV = torch.device("cuda:0")
+_cache = {}
+
+
+def pair(fam, N, M, C=3, seed=0):
+    key = ("img", fam, N, M, C, seed)
+    if key not in _cache:
+        _cache[key] = synth.make_pair(fam, N, M, C, seed)
+    return _cache[key]
+
+
+def oracle_E(fam, N, M, C=3, seed=0):
+    key = ("E", fam, N, M, C, seed)
+    if key not in _cache:
+        I, T = pair(fam, N, M, C, seed)
+        _cache[key] = oracle.error_matrix(I, T, M)
+    return _cache[key]
+
+
+def dev(x):
+    return torch.from_numpy(np.ascontiguousarray(x)).to(DEV)
+
+
+# shapes: (N, M, C) -- BASELINE configs 1-3 plus ragged / odd-S / grayscale cases
+SHAPES = [(128, 8, 3), (512, 16, 3), (90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (64, 64, 1), (30, 10, 3)]
+
+
+# ------------------------------------------------------------------ Step 1 --
+@pytest.mark.parametrize("N,M,C", SHAPES)
+def test_pack_tiles_parity(N, M, C):
+    I, _ = pair("noise", N, M, C)
+    got = pm.pack_tiles(dev(I), M).cpu().numpy()
+    assert (got == oracle.tiles(I, M)).all()
+
+
+# ------------------------------------------------------------------ Step 2 --
+@pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
+@pytest.mark.parametrize("N,M,C", SHAPES)
+def test_error_matrix_parity(fam, N, M, C):
+    I, T = pair(fam, N, M, C)
+    E = pm.error_matrix(dev(I), dev(T), M).cpu().numpy()
+    assert (E == oracle_E(fam, N, M, C)).all()
+
+
+def test_error_matrix_config3_full():
+    # n = 4096, no split-K path, 32 x 32 CTA tiles
+    E = pm.error_matrix(*map(dev, pair("smooth", 1024, 16)), 16).cpu().numpy()
+    assert (E == oracle_E("smooth", 1024, 16)).all()
+
+
+@pytest.mark.parametrize("rows", [(0, 1), (5, 77), (128, 256), (255, 256), (40, 40)])
+def test_error_matrix_row_shards(rows):
+    I, T = pair("smooth", 128, 8)
+    part = pm.error_matrix(dev(I), dev(T), 8, rows=rows).cpu().numpy()
+    assert (part == oracle_E("smooth", 128, 8)[rows[0]:rows[1]]).all()
+
+
+def test_error_matrix_padded_ld():
+    I, T = pair("smooth", 128, 8)
+    big = torch.full((256, 300), -7, dtype=torch.int32, device=DEV)
+    pm.error_matrix(dev(I), dev(T), 8, out=big[:, :256])
+    got = big.cpu().numpy()
+    assert (got[:, :256] == oracle_E("smooth", 128, 8)).all()
+    assert (got[:, 256:] == -7).all(), "writes stay inside [0, S) of each row"
+
+
+def test_error_matrix_extremes():
+    # black vs white: every entry 255 * P = 195840 (max, reading R11)
+    I = np.zeros((64, 64, 3), np.uint8)
+    T = np.full((64, 64, 3), 255, np.uint8)
+    E = pm.error_matrix(dev(I), dev(T), 16).cpu().numpy()
+    assert (E == 255 * 768).all()
+
+
+def test_error_matrix_from_tiles():
+    I, T = pair("smooth", 512, 16)
+    It, Tt = pm.pack_tiles(dev(I), 16), pm.pack_tiles(dev(T), 16)
+    E = pm.error_matrix_tiles(It, Tt, 768).cpu().numpy()
+    assert (E == oracle_E("smooth", 512, 16)).all()
+
+
+def _sampled_E_check(I, T, M, Egpu_rows, row0, rng, k):
+    n_rows, S = Egpu_rows.shape
+    us = rng.integers(0, n_rows, size=k)
+    vs = rng.integers(0, S, size=k)
+    got = Egpu_rows[torch.from_numpy(us).to(DEV), torch.from_numpy(vs).to(DEV)].cpu().numpy()
+    for u, v, g in zip(us, vs, got):
+        assert g == oracle.error_entry(I, T, M, row0 + int(u), int(v)), (row0 + u, v)
+
+
+def test_error_matrix_config4_sampled():
+    I, T = pair("smooth", 2048, 16)
+    E = pm.error_matrix(dev(I), dev(T), 16)
+    rng = np.random.default_rng(4)
+    _sampled_E_check(I, T, 16, E, 0, rng, 3000)
+    # the four corners and the diagonal ends explicitly
+    for u, v in [(0, 0), (0, 16383), (16383, 0), (16383, 16383)]:
+        assert int(E[u, v]) == oracle.error_entry(I, T, 16, u, v)
+
+
+def test_error_matrix_config5_row_chunks_sampled():
+    # n = 65536 (16 GiB E): computed in 4096-row shards, as a rank of an 8-GPU
+    # job would, each shard sampled against the oracle
+    I, T = pair("smooth", 4096, 16)
+    dI, dT = dev(I), dev(T)
+    rng = np.random.default_rng(5)
+    buf = torch.empty((4096, 65536), dtype=torch.int32, device=DEV)
+    for r0 in range(0, 65536, 4096):
+        pm.error_matrix(dI, dT, 16, rows=(r0, r0 + 4096), out=buf)
+        _sampled_E_check(I, T, 16, buf, r0, rng, 150)
+
+
+# ------------------------------------------------------------------ Alg. 2 --
+def _check_ls(E_np, method, perm0=None, max_rounds=0):
+    ref = oracle.local_search(E_np, r0=perm0, max_rounds=max_rounds)
+    E = dev(E_np)
+    perm = dev(np.arange(E_np.shape[0], dtype=np.int32) if perm0 is None else perm0.astype(np.int32))
+    out, rounds, swaps, per, st = pm.local_search(E, perm, max_rounds=max_rounds, method=method,
+                                                  allow_not_converged=True)
+    assert (out.cpu().numpy() == ref[0]).all(), "final rearrangement r"
+    assert (rounds, swaps) == (ref[1], ref[2])
+    assert (per == ref[3][: len(per)]).all()
+    assert st == ref[4]
+    return ref
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "shuffle", "transposition", "identical"])
+def test_local_search_parity_config1(method, fam):
+    _check_ls(oracle_E(fam, 128, 8), method)
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
+def test_local_search_parity_config2(method, fam):
+    _check_ls(oracle_E(fam, 512, 16), method)
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+def test_local_search_parity_config3(method):
+    ref = _check_ls(oracle_E("smooth", 1024, 16), method)
+    assert ref[1] >= 3
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("N,M,C", [(90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (30, 10, 3), (64, 64, 1)])
+def test_local_search_parity_ragged_and_odd(method, N, M, C):
+    # S = 81, 49, 9 are odd (the fixed point idles, reading R9); S = 1 trivial
+    _check_ls(oracle_E("smooth", N, M, C), method)
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+def test_local_search_resume_from_any_bijection(method):
+    E = oracle_E("noise", 128, 8)
+    rng = np.random.default_rng(3)
+    _check_ls(E, method, perm0=rng.permutation(256).astype(np.int32))
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+def test_local_search_max_rounds_then_resume(method):
+    E_np = oracle_E("smooth", 512, 16)
+    ref = _check_ls(E_np, method, max_rounds=2)
+    assert ref[4] == pm.PM_ERR_NOT_CONVERGED
+    _check_ls(E_np, method, perm0=ref[0])
+
+
+@pytest.mark.parametrize("method", ["cta", "class"])
+def test_local_search_rejects_non_permutation(method):
+    E = dev(oracle_E("smooth", 128, 8))
+    bad = torch.arange(256, dtype=torch.int32, device=DEV)
+    bad[7] = 3
+    with pytest.raises(pm.PMError) as ei:
+        pm.local_search(E, bad, method=method)
+    assert ei.value.status == pm.PM_ERR_NOT_PERMUTATION
+    bad[7] = 999
+    with pytest.raises(pm.PMError) as ei:
+        pm.local_search(E, bad, method=method)
+    assert ei.value.status == pm.PM_ERR_NOT_PERMUTATION
+
+
+def test_local_search_random_small_matrices():
+    # tie-heavy random E for S <= 9 against the oracle replay, both methods
+    rng = np.random.default_rng(0)
+    for _ in range(25):
+        S = int(rng.integers(1, 10))
+        E = rng.integers(0, 4, size=(S, S)).astype(np.int32)
+        for method in ("cta", "class"):
+            _check_ls(E, method)
+
+
+def _two_opt_gpu(E, perm):
+    F = E.index_select(0, perm.long())                   # F[u][v] = E[r[u]][v]
+    d = torch.diagonal(F).to(torch.int64)
+    S = F.shape[0]
+    for r0 in range(0, S, 2048):
+        r1 = min(S, r0 + 2048)
+        lhs = d[r0:r1, None] + d[None, :]
+        rhs = F[r0:r1].to(torch.int64) + F[:, r0:r1].T.to(torch.int64)
+        if bool((lhs > rhs).any()):
+            return False
+    return True
+
+
+def test_local_search_config4_properties_and_closed_form():
+    # n = 16384 (E = 1 GiB, beyond L2): transposition closed form (1 swap,
+    # 2 rounds, cost 0) and, on the smooth family, bijection + 2-opt + cost.
+    I, T = pair("transposition", 2048, 16)
+    E = pm.error_matrix(dev(I), dev(T), 16)
+    moved = torch.nonzero(torch.diagonal(E)).flatten().cpu().numpy()
+    assert len(moved) == 2
+    perm, rounds, swaps, per, st = pm.local_search(E)
+    expect = np.arange(16384)
+    expect[moved[0]], expect[moved[1]] = moved[1], moved[0]
+    assert (perm.cpu().numpy() == expect).all() and (rounds, swaps) == (2, 1)
+    assert pm.cost(E, perm) == 0
+
+    I, T = pair("smooth", 2048, 16)
+    E = pm.error_matrix(dev(I), dev(T), 16)
+    perm, rounds, swaps, per, st = pm.local_search(E)
+    p = perm.cpu().numpy()
+    assert sorted(p.tolist()) == list(range(16384))
+    assert per[-1] == 0 and per.sum() == swaps
+    assert _two_opt_gpu(E, perm)
+    assert pm.cost(E, perm) == int(E[perm.long(), torch.arange(16384, device=DEV)].to(torch.int64).sum())
+
+
+# ------------------------------------------------------------------ Eq. (2) -
+@pytest.mark.parametrize("N,M,C", [(128, 8, 3), (512, 16, 3), (90, 10, 3)])
+def test_cost_parity(N, M, C):
+    E_np = oracle_E("smooth", N, M, C)
+    S = E_np.shape[0]
+    rng = np.random.default_rng(S)
+    for perm in (np.arange(S), rng.permutation(S)):
+        perm = perm.astype(np.int32)
+        assert pm.cost(dev(E_np), dev(perm)) == oracle.cost(E_np, perm)
+
+
+def test_cost_int64():
+    S = 64
+    E = torch.full((S, S), 2**31 - 1, dtype=torch.int32, device=DEV)
+    assert pm.cost(E, torch.arange(S, dtype=torch.int32, device=DEV)) == S * (2**31 - 1)
+
+
+# -------------------------------------------------------------- pipeline ----
+@pytest.mark.parametrize("method", ["auto", "cta", "class"])
+def test_photomosaic_pipeline_config2(method):
+    I, T = pair("smooth", 512, 16)
+    E_np = oracle_E("smooth", 512, 16)
+    ref = oracle.local_search(E_np)
+    perm, rounds, swaps, c, E = pm.photomosaic(dev(I), dev(T), 16, method=method)
+    assert (E.cpu().numpy() == E_np).all()
+    assert (perm.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    assert c == oracle.cost(E_np, ref[0])
+
+
+def test_photomosaic_host_config1():
+    I, T = pair("smooth", 128, 8)
+    E_np = oracle_E("smooth", 128, 8)
+    ref = oracle.local_search(E_np)
+    perm, rounds, swaps, c = pm.photomosaic_host(I, T, 8)
+    assert (perm == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    assert c == oracle.cost(E_np, ref[0])
+
+
+# ------------------------------------------------------------ error paths ---
+def test_invalid_arguments_launch_nothing():
+    L = pm.lib()
+    I = torch.zeros((64, 64, 3), dtype=torch.uint8, device=DEV)
+    E = torch.zeros((16, 16), dtype=torch.int32, device=DEV)
+    n0 = pm.launch_count()
+    assert L.pm_error_matrix(I.data_ptr(), I.data_ptr(), 64, 15, 3, 0, 16, E.data_ptr(), 16, None) == pm.PM_ERR_INVALID
+    assert L.pm_error_matrix(I.data_ptr(), I.data_ptr(), 64, 16, 3, 0, 17, E.data_ptr(), 16, None) == pm.PM_ERR_INVALID
+    assert L.pm_error_matrix(I.data_ptr(), I.data_ptr(), 64, 16, 3, 0, 16, E.data_ptr(), 15, None) == pm.PM_ERR_INVALID
+    assert L.pm_error_matrix(None, I.data_ptr(), 64, 16, 3, 0, 16, E.data_ptr(), 16, None) == pm.PM_ERR_INVALID
+    # 255 * P must fit int32 (reading R11)
+    assert L.pm_error_matrix(I.data_ptr(), I.data_ptr(), 8192, 4096, 1, 0, 4, E.data_ptr(), 16,
+                             None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search(E.data_ptr(), 15, 16, E.data_ptr(), 0, None, None, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_ex(E.data_ptr(), 16, 16, E.data_ptr(), 0, 9, None, None, None, 0,
+                                None) == pm.PM_ERR_INVALID
+    assert L.pm_cost(E.data_ptr(), 16, 0, E.data_ptr(), None, None) == pm.PM_ERR_INVALID
+    assert pm.launch_count() == n0
+
+
+def test_launch_count_increments():
+    I, T = pair("smooth", 128, 8)
+    n0 = pm.launch_count()
+    pm.photomosaic(dev(I), dev(T), 8, method="cta")
+    assert pm.launch_count() - n0 >= 5   # 2 pack + E + iota + search + cost
