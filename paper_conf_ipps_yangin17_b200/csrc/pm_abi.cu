@@ -107,10 +107,11 @@ pm_status_t pm_pack_tiles(const uint8_t* d_img, int32_t N, int32_t M, int32_t C,
 pm_status_t pm_error_matrix_tiles(const uint8_t* d_input_tiles, const uint8_t* d_target_tiles,
                                   int64_t ld_tiles, int32_t S, int32_t P, int32_t row_begin, int32_t row_end,
                                   int32_t* d_E, int64_t ld_E, pm_stream_t stream) {
-  if (!d_input_tiles || !d_target_tiles || !d_E) return PM_ERR_INVALID;
   if (S < 1 || P < 1 || (int64_t)P * 255 > INT32_MAX) return PM_ERR_INVALID;
   if (ld_tiles < P || ld_tiles % 64 != 0) return PM_ERR_INVALID;
   if (row_begin < 0 || row_end > S || row_begin > row_end || ld_E < S) return PM_ERR_INVALID;
+  if (row_begin == row_end) return PM_OK;
+  if (!d_input_tiles || !d_target_tiles || !d_E) return PM_ERR_INVALID;
   PM_CUDA_TRY(launch_sad(d_input_tiles + (int64_t)row_begin * ld_tiles, d_target_tiles, ld_tiles,
                          row_end - row_begin, S, P, d_E, ld_E, (cudaStream_t)stream));
   return PM_OK;
@@ -119,11 +120,12 @@ pm_status_t pm_error_matrix_tiles(const uint8_t* d_input_tiles, const uint8_t* d
 pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M, int32_t C,
                             int32_t row_begin, int32_t row_end, int32_t* d_E, int64_t ld_E,
                             pm_stream_t stream) {
-  if (!d_input || !d_target || !d_E || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  if (!valid_image_args(N, M, C)) return PM_ERR_INVALID;
   const int32_t g = N / M;
   const int32_t S = g * g;
   if (row_begin < 0 || row_end > S || row_begin > row_end || ld_E < S) return PM_ERR_INVALID;
-  if (row_begin == row_end) return PM_OK;
+  if (row_begin == row_end) return PM_OK;   // empty shard: nothing to do, pointers unused
+  if (!d_input || !d_target || !d_E) return PM_ERR_INVALID;
   cudaStream_t st = (cudaStream_t)stream;
   const int64_t ldt = pm_tile_stride(M, C);
   const int32_t nrows = row_end - row_begin;

@@ -91,6 +91,9 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
                              int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
                              int32_t* used_method);
 int32_t ls_class_launches_per_round(int32_t S);
+int32_t ls_window_max_S();
+pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                       LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm,
                         int64_t* d_cost, cudaStream_t st);
 

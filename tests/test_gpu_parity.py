@@ -144,39 +144,39 @@ def _check_ls(E_np, method, perm0=None, max_rounds=0):
     return ref
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "shuffle", "transposition", "identical"])
 def test_local_search_parity_config1(method, fam):
     _check_ls(oracle_E(fam, 128, 8), method)
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
 def test_local_search_parity_config2(method, fam):
     _check_ls(oracle_E(fam, 512, 16), method)
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 def test_local_search_parity_config3(method):
     ref = _check_ls(oracle_E("smooth", 1024, 16), method)
     assert ref[1] >= 3
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 @pytest.mark.parametrize("N,M,C", [(90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (30, 10, 3), (64, 64, 1)])
 def test_local_search_parity_ragged_and_odd(method, N, M, C):
     # S = 81, 49, 9 are odd (the fixed point idles, reading R9); S = 1 trivial
     _check_ls(oracle_E("smooth", N, M, C), method)
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 def test_local_search_resume_from_any_bijection(method):
     E = oracle_E("noise", 128, 8)
     rng = np.random.default_rng(3)
     _check_ls(E, method, perm0=rng.permutation(256).astype(np.int32))
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 def test_local_search_max_rounds_then_resume(method):
     E_np = oracle_E("smooth", 512, 16)
     ref = _check_ls(E_np, method, max_rounds=2)
@@ -184,7 +184,7 @@ def test_local_search_max_rounds_then_resume(method):
     _check_ls(E_np, method, perm0=ref[0])
 
 
-@pytest.mark.parametrize("method", ["cta", "class"])
+@pytest.mark.parametrize("method", ["window", "cta", "class"])
 def test_local_search_rejects_non_permutation(method):
     E = dev(oracle_E("smooth", 128, 8))
     bad = torch.arange(256, dtype=torch.int32, device=DEV)
@@ -204,7 +204,7 @@ def test_local_search_random_small_matrices():
     for _ in range(25):
         S = int(rng.integers(1, 10))
         E = rng.integers(0, 4, size=(S, S)).astype(np.int32)
-        for method in ("cta", "class"):
+        for method in ("window", "cta", "class"):
             _check_ls(E, method)
 
 
@@ -262,7 +262,7 @@ def test_cost_int64():
 
 
 # -------------------------------------------------------------- pipeline ----
-@pytest.mark.parametrize("method", ["auto", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "window", "cta", "class"])
 def test_photomosaic_pipeline_config2(method):
     I, T = pair("smooth", 512, 16)
     E_np = oracle_E("smooth", 512, 16)
@@ -307,3 +307,15 @@ def test_launch_count_increments():
     n0 = pm.launch_count()
     pm.photomosaic(dev(I), dev(T), 8, method="cta")
     assert pm.launch_count() - n0 >= 5   # 2 pack + E + iota + search + cost
+
+
+@pytest.mark.parametrize("N,M", [(1600, 40), (1150, 25), (1344, 24), (2048, 32)])
+def test_local_search_window_sizes(N, M):
+    # S = 1600 and 2116 (K = 16 window), 3136 and 4096 (K = 8 window), grayscale noise
+    _check_ls(oracle_E("noise", N, M, 1), "window")
+
+
+@pytest.mark.parametrize("S_side", [33, 45, 63])
+def test_local_search_window_odd_mid(S_side):
+    # odd S between the window tiers (1089, 2025, 3969)
+    _check_ls(oracle_E("smooth", S_side * 4, 4, 3), "window")
