@@ -165,7 +165,7 @@ static pm_status_t run_class(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
     cg = it->second;
   }
   int32_t* scratch = nullptr;   // d [S] + seen [S]
-  PM_CUDA_TRY(cudaMallocAsync(&scratch, sizeof(int32_t) * 2 * (size_t)(S > 0 ? S : 1), st));
+  PM_CUDA_TRY(pm::scratch_alloc(&scratch, sizeof(int32_t) * 2 * (size_t)(S > 0 ? S : 1), st));
   PM_CUDA_TRY(cudaMemsetAsync(scratch + S, 0, sizeof(int32_t) * (size_t)S, st));
   LsParams hp = {};
   hp.E = E; hp.ldE = ldE; hp.r = perm; hp.d = scratch; hp.seen = scratch + S;

@@ -35,130 +35,221 @@
 
 namespace pm {
 
-constexpr int kWinThreads = 1024;
+__device__ __forceinline__ void cp_async4(int32_t* smem, const int32_t* gmem) {
+  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(d), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
-// Ep[t][pos] = E[t][(2 pos) mod m], pos in [0, m).
+// Ep[t][pos] = E[t][(2 pos) mod m] for pos in [0, m + ext): the sigma-permuted
+// row, extended cyclically by `ext` entries so that any window segment
+// [pos, pos + K + 4) can be read without wrapping.
 __global__ void k_permute_cols(const int32_t* __restrict__ E, int64_t ld, int32_t* __restrict__ Ep, int64_t ldp,
-                               int32_t S, int32_t m) {
-  const int64_t total = (int64_t)S * m;
+                               int32_t S, int32_t m, int32_t ext) {
+  const int32_t w = m + ext;
+  const int64_t total = (int64_t)S * w;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t t = i / m;
-    const int32_t pos = (int32_t)(i - t * m);
+    const int64_t t = i / w;
+    const int32_t orig = (int32_t)(i - t * w);
+    int32_t pos = orig;
+    while (pos >= m) pos -= m;
     int32_t q = 2 * pos;
     if (q >= m) q -= m;
-    Ep[t * ldp + pos] = __ldg(E + t * ld + q);
+    Ep[t * ldp + orig] = __ldg(E + t * ld + q);
   }
 }
 
-template <int K>
-struct WinSmem {
-  static constexpr int KP = K + 1;  // padded row (conflict-free column access)
-  static size_t bytes(int32_t S) { return sizeof(int32_t) * ((size_t)S * (4 + KP) + 64); }
-};
+__host__ __device__ inline int32_t win_stride(int32_t S) { return S + ((1 - S % 32) + 32) % 32; }  // == 1 mod 32
 
 template <int K>
-__global__ void __launch_bounds__(kWinThreads, 1)
+struct WinSmem {
+  static constexpr int KS = K + 4;   // stored entries per slot: an aligned superset of K
+  static size_t bytes(int32_t S) {
+    return sizeof(int32_t) * ((size_t)S * 7 + (size_t)2 * KS * win_stride(S) + 64);
+  }
+};
+
+// Per regular slot x, two windows in shared memory, stored transposed
+// (entry-major, stride SP == 1 mod 32: the slots of one class are read
+// conflict-free).  Each holds a 16-byte-aligned superset of K entries of a
+// sigma-permuted row, loaded with unconditional LDG.128 / 4 x STS; off[x] is
+// the offset of the first wanted entry inside the superset:
+//   W [off[x] + j][x] = E[r[x]][p_{wb+j}(x)]  = Ep[r[x]][sigma(1-x) + wb + j]   (class window)
+//   SW[swoff[x] + i][x] = E[r[x]][x + 2(i+1)] = Ep[r[x]][sigma(x) + i + 1]      (diagonal window)
+// Swap of regular slots (u, v) in class c = wb + j, a = r[u], b = r[v]: since
+// p_{c+i}(u) = v + 2i and p_{c+i}(v) = u + 2i,
+//   W'[j+i][u] = E[b][v+2i] = SW[i-1][v]     SW'[i-1][u] = E[b][u+2i] = W[j+i][v]
+// (and symmetrically for v): the swap is an exchange of shared-memory entries
+// with no global access.  SW' entries beyond the window are stale and are
+// reloaded at the next window (slots swapped during window w are those with
+// dgen == w) but never read before: a later swap at class c'' > c needs
+// offsets < jmax - (c'' - wb).  SW does not depend on the class, so clean
+// slots keep theirs across windows and rounds.  Slot L = S-1 walks the plain
+// row E[r[L]][u0(c)] (u0(c) = c + (m+1)/2 advances by one per class); the rare
+// swap of the fixed pair (u0, L) reloads from global.
+template <int K, int PPT, int MAXT>
+__global__ void __launch_bounds__(MAXT, 1)
 k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict__ Ep, int64_t ldp, int32_t S,
             int32_t* __restrict__ perm, int32_t max_rounds, LsResult* out, int64_t* per_round, int32_t max_log) {
-  constexpr int KP = K + 1;
-  extern __shared__ int32_t sm[];
-  int32_t* s_r = sm;               // r[x]: tile at slot x
-  int32_t* s_d = s_r + S;          // d[x] = E[r[x]][x]
-  int32_t* s_last = s_d + S;       // E[t][L] per tile t (even S)
-  int32_t* s_p0 = s_last + S;      // sigma(1 - x) per regular slot
-  int32_t* s_W = s_p0 + S;         // window [S][KP]
-  int32_t* s_ctl = s_W + (size_t)S * KP;   // [0..2] first-fire slots, [8..40] reduction
+  static_assert(K % 4 == 0, "K multiple of 4");
+  constexpr int KS = K + 4;
+  constexpr int NP = KS / 4;       // 16-byte pieces per window
+  extern __shared__ __align__(16) int32_t sm[];
+  const int32_t SP = win_stride(S);
+  int2* s_do = reinterpret_cast<int2*>(sm);   // {d[x] = E[r[x]][x], off[x]}
+  int32_t* s_r = sm + 2 * S;       // r[x]: tile at slot x
+  int32_t* s_last = s_r + S;       // E[t][L] per tile t (even S)
+  int32_t* s_sig = s_last + S;     // sigma(x)
+  int32_t* s_swoff = s_sig + S;    // offset of SW inside its superset
+  int32_t* s_dgen = s_swoff + S;   // window id of x's last swap (SW reload at the next window)
+  int32_t* s_W = s_dgen + S;       // [KS][SP]
+  int32_t* s_SW = s_W + (size_t)KS * SP;     // [KS][SP]
+  int32_t* s_ctl = s_SW + (size_t)KS * SP;   // [0..2] first-fire slots, [8..40] reduction
   const Classes cl(S);
   const int32_t m = cl.m, H = cl.half;
   const bool even = (S % 2) == 0;
   const int32_t L = S - 1;
+  const int32_t nreg = even ? S - 1 : S;       // regular slots 0..m-1
   const int tid = threadIdx.x, T = blockDim.x;
+  const int lane = tid & 31;
 
-  // ---- permutation check, then d, s_last, s_p0 ----
-  for (int32_t x = tid; x < S; x += T) s_d[x] = 0;
+  // ---- permutation check, then d, s_last, s_sig ----
+  for (int32_t x = tid; x < S; x += T) s_sig[x] = 0;
   __syncthreads();
   int bad = 0;
   for (int32_t u = tid; u < S; u += T) {
     const int32_t t = perm[u];
     s_r[u] = t;
     if (t < 0 || t >= S) bad = 1;
-    else atomicAdd(&s_d[t], 1);
+    else atomicAdd(&s_sig[t], 1);
   }
   __syncthreads();
   for (int32_t x = tid; x < S; x += T)
-    if (s_d[x] != 1) bad = 1;
+    if (s_sig[x] != 1) bad = 1;
   if (__syncthreads_or(bad)) {
     if (tid == 0) { out->status = PM_ERR_NOT_PERMUTATION; out->rounds = 0; out->swaps = 0; }
     return;
   }
   for (int32_t x = tid; x < S; x += T) {
-    s_d[x] = __ldg(E + (int64_t)s_r[x] * ld + x);
+    s_do[x] = make_int2(__ldg(E + (int64_t)s_r[x] * ld + x), 0);
     if (even) s_last[x] = __ldg(E + (int64_t)x * ld + L);
-    int32_t q = 1 - x;
-    q %= m; if (q < 0) q += m;
-    s_p0[x] = (int32_t)(((int64_t)q * H) % m);
+    const int32_t sg = (x < m) ? (int32_t)(((int64_t)x * H) % m) : 0;
+    s_sig[x] = sg;
+    s_swoff[x] = (sg + 1) & 3;
+    s_dgen[x] = -1;                   // window 0 loads every SW
   }
   if (tid < 3) s_ctl[tid] = INT32_MAX;
   __syncthreads();
 
-  // entry of slot x at class (wb + j), tile t
-  auto win_src = [&](int32_t x, int32_t t, int32_t wb, int32_t j) -> const int32_t* {
-    if (even && x == L) {
-      int32_t col = wb + j + H;
-      col %= m;
-      return E + (int64_t)t * ld + col;
-    }
-    int32_t pos = wb + j + s_p0[x];
-    pos %= m;
-    return Ep + (int64_t)t * ldp + pos;
+  auto wrap = [&](int32_t q) -> int32_t {   // q in (-m, 2m)
+    if (q < 0) q += m;
+    if (q >= m) q -= m;
+    return q;
   };
-  // reload slot x's window entries j in [j0, K) (after a swap gave it tile t)
-  auto refresh = [&](int32_t x, int32_t t, int32_t wb, int32_t j0, int32_t jmax) {
-    constexpr int CH = K < 8 ? K : 8;     // loads in flight per chunk
+  // window `wid` for classes [wb, wb + jmax): W of every slot, SW of slots
+  // swapped during window wid - 1 (and all at wid = 0)
+  auto fill = [&](int32_t wb, int32_t jmax, int32_t wid) {
+    constexpr int U = MAXT <= 512 ? 4 : 2;   // loads in flight per thread
+    __syncthreads();
+    const int32_t total = nreg * NP;
+    for (int32_t f0 = 0; f0 < total; f0 += U * T) {
+      int4 val[U];
+      int32_t dst[U];
 #pragma unroll
-    for (int jc = 0; jc < K; jc += CH) {
-      if (jc + CH <= j0 || jc >= jmax) continue;
-      int32_t v[CH];
-#pragma unroll
-      for (int q = 0; q < CH; ++q) {
-        const int j = jc + q;
-        if (j >= j0 && j < jmax) v[q] = __ldg(win_src(x, t, wb, j));
+      for (int uu = 0; uu < U; ++uu) {
+        const int32_t f = f0 + uu * T + tid;
+        dst[uu] = -1;
+        if (f < total) {
+          const int32_t x = f / NP, q = f - x * NP;
+          const int32_t pos = wrap(wb + H - s_sig[x]);
+          const int32_t base = pos & ~3;
+          val[uu] = __ldg(reinterpret_cast<const int4*>(Ep + (int64_t)s_r[x] * ldp + base) + q);
+          if (q == 0) s_do[x].y = pos - base;
+          dst[uu] = (4 * q) * SP + x;
+        }
       }
 #pragma unroll
-      for (int q = 0; q < CH; ++q) {
-        const int j = jc + q;
-        if (j >= j0 && j < jmax) s_W[x * KP + j] = v[q];
+      for (int uu = 0; uu < U; ++uu) {
+        if (dst[uu] < 0) continue;
+        int32_t* w = s_W + dst[uu];
+        w[0] = val[uu].x; w[SP] = val[uu].y; w[2 * SP] = val[uu].z; w[3 * SP] = val[uu].w;
       }
     }
+    for (int32_t f0 = 0; f0 < total; f0 += U * T) {
+      int4 val[U];
+      int32_t dst[U];
+#pragma unroll
+      for (int uu = 0; uu < U; ++uu) {
+        const int32_t f = f0 + uu * T + tid;
+        dst[uu] = -1;
+        if (f < total) {
+          const int32_t x = f / NP, q = f - x * NP;
+          if (s_dgen[x] == wid - 1) {
+            const int32_t base = (s_sig[x] + 1) & ~3;
+            val[uu] = __ldg(reinterpret_cast<const int4*>(Ep + (int64_t)s_r[x] * ldp + base) + q);
+            dst[uu] = (4 * q) * SP + x;
+          }
+        }
+      }
+#pragma unroll
+      for (int uu = 0; uu < U; ++uu) {
+        if (dst[uu] < 0) continue;
+        int32_t* w = s_SW + dst[uu];
+        w[0] = val[uu].x; w[SP] = val[uu].y; w[2 * SP] = val[uu].z; w[3 * SP] = val[uu].w;
+      }
+    }
+    if (even) {
+      for (int32_t j = tid; j < jmax; j += T) s_W[j * SP + L] = __ldg(E + (int64_t)s_r[L] * ld + wrap(wb + j + H));
+      if (tid == 0) s_do[L].y = 0;
+    }
+    __syncthreads();
   };
-  // evaluate pair k of class cc (window offset j); returns fire
-  auto eval = [&](int32_t cc, int32_t k, int32_t j, int32_t& u, int32_t& v, int32_t& ou, int32_t& ov) -> bool {
-    cl.pair(cc, k, u, v);
-    if (even && k == 0) ou = s_last[s_r[u]];       // u = u0(cc), partner L
-    else ou = s_W[u * KP + j];
-    ov = s_W[v * KP + j];
-    return (int64_t)s_d[u] + s_d[v] > (int64_t)ou + ov;
+
+  // this thread's pairs k = tid + q*T; (u, v) tracked for the current class
+  int32_t pu[PPT] = {}, pv[PPT] = {};
+  auto set_class = [&](int32_t c) {
+#pragma unroll
+    for (int q = 0; q < PPT; ++q) {
+      const int32_t k = tid + q * T;
+      if (k < cl.npairs) cl.pair(c, k, pu[q], pv[q]);
+    }
+  };
+  auto advance = [&](int32_t delta) {   // classes are consecutive: u0 + k, u0 - k, u0 all shift by +1
+#pragma unroll
+    for (int q = 0; q < PPT; ++q) {
+      const int32_t k = tid + q * T;
+      int32_t a = pu[q] + delta; if (a >= m) a -= m;
+      pu[q] = a;
+      if (!(even && k == 0)) { int32_t b = pv[q] + delta; if (b >= m) b -= m; pv[q] = b; }
+    }
+  };
+  // O(u), O(v) at window offset j; fire iff d[u] + d[v] > O(u) + O(v)
+  auto eval = [&](int q, int32_t u, int32_t v, int32_t j, int2& du, int2& dv, int32_t& ou, int32_t& ov) -> bool {
+    const int32_t k = tid + q * T;
+    du = s_do[u];
+    dv = s_do[v];
+    if (even && k == 0) ou = s_last[s_r[u]];          // u = u0(c), partner L
+    else ou = s_W[(j + du.y) * SP + u];
+    ov = s_W[(j + dv.y) * SP + v];
+    return (int64_t)du.x + dv.x > (int64_t)ou + ov;
   };
 
   int32_t rounds = 0;
   int64_t total = 0;
   int status = PM_OK;
   uint32_t batch = 0;
+  int32_t wid = 0;
   int32_t B = 1;
   for (;;) {                                           // Alg. 2 line 1
     int mysw = 0;
     int32_t c = 0;
     int32_t wb = INT32_MIN / 2;
+    set_class(0);
     while (c < cl.ncls) {                              // line 3, classes in order
-      if (c >= wb + K) {                               // stream the next window
+      if (c >= wb + K) {
         wb = c;
-        const int32_t jmax = min(K, cl.ncls - wb);
-        __syncthreads();
-        for (int32_t f = tid; f < S * K; f += T) {
-          const int32_t x = f / K, j = f - x * K;
-          if (j < jmax) s_W[x * KP + j] = __ldg(win_src(x, s_r[x], wb, j));
-        }
-        __syncthreads();
+        fill(wb, min(K, cl.ncls - wb), wid);
+        ++wid;
       }
       const int32_t jmax = min(K, cl.ncls - wb);
       int32_t* first_slot = s_ctl + (batch % 3);
@@ -166,49 +257,93 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
       ++batch;
       const int32_t cend = min(c + B, wb + jmax);
       int32_t cc = c;
-      bool apply = true;
       if (cend - c > 1) {
         // speculative: all pairs of classes [c, cend) on the current state
         const int32_t nb = cend - c;
-        const int32_t items = nb * cl.npairs;
-        for (int32_t it = tid; it < items; it += T) {
-          const int32_t jj = it / cl.npairs, k = it - jj * cl.npairs;
-          int32_t u, v, ou, ov;
-          if (eval(c + jj, k, c + jj - wb, u, v, ou, ov)) atomicMin(first_slot, jj);
+#pragma unroll
+        for (int q = 0; q < PPT; ++q) {
+          if (tid + q * T >= cl.npairs) continue;
+          int32_t u = pu[q], v = pv[q];
+          const bool special = even && tid + q * T == 0;
+          for (int32_t jj = 0; jj < nb; ++jj) {
+            int2 du, dv;
+            int32_t ou, ov;
+            if (eval(q, u, v, c + jj - wb, du, dv, ou, ov)) { atomicMin(first_slot, jj); break; }
+            u = (u + 1 == m) ? 0 : u + 1;
+            if (!special) v = (v + 1 == m) ? 0 : v + 1;
+          }
         }
         __syncthreads();
         const int32_t first = *first_slot;
         if (first == INT32_MAX) {
+          advance(nb);
           c = cend;
           B = min(2 * B, K);
-          apply = false;
-        } else {
-          cc = c + first;
-          B = first == 0 ? 1 : first;
+          continue;
         }
+        advance(first);
+        cc = c + first;
+        B = first == 0 ? 1 : first;
       }
-      if (apply) {
-        // exact step of class cc: evaluate, swap (line 6), refresh windows
-        const int32_t j = cc - wb;
-        int fired = 0;
-        for (int32_t k = tid; k < cl.npairs; k += T) {
-          int32_t u, v, ou, ov;
-          if (eval(cc, k, j, u, v, ou, ov)) {
-            const int32_t a = s_r[u], b = s_r[v];
-            s_r[u] = b; s_r[v] = a;
-            s_d[u] = ov; s_d[v] = ou;      // d[u] = E[b][u] = O(v), d[v] = E[a][v] = O(u)
-            ++mysw;
-            fired = 1;
-            if (j + 1 < jmax) {
-              refresh(u, b, wb, j + 1, jmax);
-              refresh(v, a, wb, j + 1, jmax);
+      // exact step of class cc: evaluate, swap (line 6), exchange windows
+      const int32_t j = cc - wb;
+      int fired = 0;
+#pragma unroll
+      for (int q = 0; q < PPT; ++q) {                  // warp-uniform
+        const int32_t k = tid + q * T;
+        const int32_t u = pu[q], v = pv[q];
+        int32_t a = 0, b = 0;
+        int2 du, dv;
+        int32_t ou = 0, ov = 0;
+        bool f = false;
+        if (k < cl.npairs && eval(q, u, v, j, du, dv, ou, ov)) {
+          a = s_r[u]; b = s_r[v];
+          s_r[u] = b; s_r[v] = a;
+          s_do[u].x = ov; s_do[v].x = ou;  // d[u] = E[b][u] = O(v), d[v] = E[a][v] = O(u)
+          s_dgen[u] = wid - 1; s_dgen[v] = wid - 1;
+          ++mysw;
+          fired = 1;
+          f = true;
+        }
+        unsigned mask = __ballot_sync(0xffffffffu, f);
+        while (mask) {
+          const int sl = __ffs(mask) - 1;
+          mask &= mask - 1;
+          const int32_t su = __shfl_sync(0xffffffffu, u, sl), sv = __shfl_sync(0xffffffffu, v, sl);
+          const bool sfixed = even && (__shfl_sync(0xffffffffu, k, sl) == 0);
+          const int32_t ofu = s_do[su].y, ofv = s_do[sv].y;
+          if (!sfixed) {
+            const int32_t swu = s_swoff[su], swv = s_swoff[sv];
+            for (int32_t jj = j + 1 + lane; jj < jmax; jj += 32) {
+              const int32_t i = jj - j - 1;
+              int32_t* Wu = s_W + (jj + ofu) * SP + su;
+              int32_t* Wv = s_W + (jj + ofv) * SP + sv;
+              int32_t* Xu = s_SW + (i + swu) * SP + su;
+              int32_t* Xv = s_SW + (i + swv) * SP + sv;
+              const int32_t wu = *Wu, wv = *Wv, xu = *Xu, xv = *Xv;
+              *Wu = xv; *Xu = wv;
+              *Wv = xu; *Xv = wu;
+            }
+          } else {
+            // (u0, L): u0 now holds b (walks Ep[b][sigma(u0) + i]), L holds a
+            // (walks E[a][u0 + i]); reload from global (rare: 1 pair per class)
+            const int32_t sa = __shfl_sync(0xffffffffu, a, sl), sb = __shfl_sync(0xffffffffu, b, sl);
+            const int32_t sg = s_sig[su], swu = s_swoff[su];
+            for (int32_t jj = j + 1 + lane; jj < jmax; jj += 32) {
+              const int32_t i = jj - j;
+              const int32_t e1 = __ldg(Ep + (int64_t)sb * ldp + sg + i);
+              const int32_t e2 = __ldg(E + (int64_t)sa * ld + wrap(su + i));
+              s_W[(jj + ofu) * SP + su] = e1;
+              s_SW[(i - 1 + swu) * SP + su] = e1;
+              s_W[(jj + ofv) * SP + sv] = e2;
             }
           }
         }
-        const int any = __syncthreads_or(fired);
-        if (cend - c <= 1 && !any) B = 2;               // quiet class: start speculating
-        c = cc + 1;
       }
+      const int any = __syncthreads_or(fired);
+      if (cend - c <= 1 && !any) B = 2;                 // quiet class: start speculating
+      advance(1);
+      c = cc + 1;
     }
     // round end: count swaps (line 7 / 11)
     int sw = mysw;
@@ -216,7 +351,7 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     for (int o = 16; o > 0; o >>= 1) sw += __shfl_xor_sync(0xffffffffu, sw, o);
     int* red = s_ctl + 8;
     __syncthreads();
-    if ((tid & 31) == 0) red[tid >> 5] = sw;
+    if (lane == 0) red[tid >> 5] = sw;
     __syncthreads();
     int rs = 0;
     for (int w = 0; w < (T >> 5); ++w) rs += red[w];
@@ -232,9 +367,9 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
   if (tid == 0) { out->status = status; out->rounds = rounds; out->swaps = total; }
 }
 
-int32_t ls_window_max_S() { return 4096; }
+int32_t ls_window_max_S() { return 2048; }
 
-template <int K>
+template <int K, int PPT, int MAXT>
 static pm_status_t launch_window_k(const int32_t* E, int64_t ldE, const int32_t* Ep, int64_t ldp, int32_t S,
                                    int32_t* perm, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
                                    int32_t max_log, cudaStream_t st) {
@@ -243,10 +378,13 @@ static pm_status_t launch_window_k(const int32_t* E, int64_t ldE, const int32_t*
   PM_CUDA_TRY(cudaGetDevice(&dev));
   PM_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   if (smem > (size_t)optin) return PM_ERR_UNSUPPORTED;
-  PM_CUDA_TRY(cudaFuncSetAttribute(k_ls_window<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int threads = kWinThreads;
-  while (threads > 64 && threads / 2 >= S / 2) threads /= 2;
-  k_ls_window<K><<<1, threads, smem, st>>>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log);
+  PM_CUDA_TRY(cudaFuncSetAttribute(k_ls_window<K, PPT, MAXT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int32_t npairs = S / 2;
+  int threads = (npairs + PPT - 1) / PPT;
+  threads = (threads + 31) / 32 * 32;
+  if (threads < 32) threads = 32;
+  if (threads > MAXT) return PM_ERR_UNSUPPORTED;
+  k_ls_window<K, PPT, MAXT><<<1, threads, smem, st>>>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log);
   note_launch();
   PM_CUDA_TRY(cudaGetLastError());
   return PM_OK;
@@ -257,22 +395,22 @@ pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, 
   if (S > ls_window_max_S()) return PM_ERR_UNSUPPORTED;
   const Classes cl(S);
   const int32_t m = cl.m;
-  const int64_t ldp = ((int64_t)m + 31) / 32 * 32;
+  const int32_t ext = 16 + 8;                                   // >= K + 4 for every K used
+  const int64_t ldp = ((int64_t)m + ext + 31) / 32 * 32;
   int32_t* Ep = nullptr;
-  PM_CUDA_TRY(cudaMallocAsync(&Ep, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
+  PM_CUDA_TRY(pm::scratch_alloc(&Ep, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
   {
-    const int64_t total = (int64_t)S * m;
+    const int64_t total = (int64_t)S * (m + ext);
     int64_t blocks = (total + 255) / 256;
     if (blocks > 148 * 8) blocks = 148 * 8;
     if (blocks < 1) blocks = 1;
-    k_permute_cols<<<(unsigned)blocks, 256, 0, st>>>(E, ldE, Ep, ldp, S, m);
+    k_permute_cols<<<(unsigned)blocks, 256, 0, st>>>(E, ldE, Ep, ldp, S, m, ext);
     note_launch();
     PM_CUDA_TRY(cudaGetLastError());
   }
   pm_status_t s;
-  if (S <= 1024) s = launch_window_k<32>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
-  else if (S <= 2048) s = launch_window_k<16>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
-  else s = launch_window_k<8>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+  if (S <= 1024) s = launch_window_k<16, 1, 512>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+  else s = launch_window_k<4, 1, 1024>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
   PM_CUDA_TRY(cudaFreeAsync(Ep, st));
   return s;
 }

@@ -8,8 +8,34 @@
 
 #include "pm_internal.cuh"
 
+#include <mutex>
+
 namespace pm {
 std::atomic<int64_t> g_launches{0};
+
+cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
+  static std::mutex mu;
+  static cudaMemPool_t pools[64] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  cudaMemPool_t pool;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (!pools[dev]) {
+      cudaMemPoolProps props = {};
+      props.allocType = cudaMemAllocationTypePinned;
+      props.location.type = cudaMemLocationTypeDevice;
+      props.location.id = dev;
+      if ((e = cudaMemPoolCreate(&pools[dev], &props)) != cudaSuccess) return e;
+      uint64_t thr = UINT64_MAX;
+      if ((e = cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &thr)) != cudaSuccess) return e;
+    }
+    pool = pools[dev];
+  }
+  return cudaMallocFromPoolAsync(p, bytes, pool, st);
+}
 }  // namespace pm
 
 using namespace pm;
@@ -48,7 +74,7 @@ pm_status_t local_search_impl(const int32_t* d_E, int64_t ld_E, int32_t S, int32
   DevBuf buf;
   buf.st = st;
   const size_t bytes = sizeof(LsResult) + sizeof(int64_t) * kMaxLog;
-  PM_CUDA_TRY(cudaMallocAsync(&buf.p, bytes, st));
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, bytes, st));
   LsResult* dres = reinterpret_cast<LsResult*>(buf.p);
   int64_t* dlog = reinterpret_cast<int64_t*>(reinterpret_cast<char*>(buf.p) + sizeof(LsResult));
   PM_CUDA_TRY(cudaMemsetAsync(buf.p, 0, bytes, st));
@@ -131,7 +157,7 @@ pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target, int
   const int32_t nrows = row_end - row_begin;
   DevBuf buf;
   buf.st = st;
-  PM_CUDA_TRY(cudaMallocAsync(&buf.p, (size_t)ldt * ((size_t)nrows + S), st));
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, (size_t)ldt * ((size_t)nrows + S), st));
   uint8_t* tI = reinterpret_cast<uint8_t*>(buf.p);
   uint8_t* tT = tI + (size_t)ldt * nrows;
   PM_CUDA_TRY(launch_pack(d_input, N, M, C, tI, ldt, row_begin, row_end, st));
@@ -202,7 +228,7 @@ pm_status_t pm_cost(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* 
   cudaStream_t st = (cudaStream_t)stream;
   DevBuf buf;
   buf.st = st;
-  PM_CUDA_TRY(cudaMallocAsync(&buf.p, sizeof(int64_t), st));
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, sizeof(int64_t), st));
   pm_status_t s = pm_cost_async(d_E, ld_E, S, d_perm, reinterpret_cast<int64_t*>(buf.p), stream);
   if (s != PM_OK) return s;
   PM_CUDA_TRY(cudaMemcpyAsync(h_cost, buf.p, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
@@ -241,7 +267,7 @@ pm_status_t pm_photomosaic(const uint8_t* d_input, const uint8_t* d_target, int3
   DevBuf buf;   // {status, rounds, swaps, cost}
   buf.st = st;
   if (!d_input || !d_target || !d_E || !d_perm || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
-  PM_CUDA_TRY(cudaMallocAsync(&buf.p, 4 * sizeof(int64_t), st));
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, 4 * sizeof(int64_t), st));
   pm_status_t s = pm_photomosaic_async(d_input, d_target, N, M, C, d_E, ld_E, d_perm, method,
                                        reinterpret_cast<int64_t*>(buf.p), stream);
   if (s != PM_OK) return s;
@@ -265,7 +291,7 @@ pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
   const size_t bytes = 2 * img + sizeof(int32_t) * (size_t)S * (size_t)S + sizeof(int32_t) * (size_t)S + 64;
   DevBuf buf;
   buf.st = st;
-  PM_CUDA_TRY(cudaMallocAsync(&buf.p, bytes, st));
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, bytes, st));
   char* base = reinterpret_cast<char*>(buf.p);
   int32_t* dE = reinterpret_cast<int32_t*>(base);
   int32_t* dperm = dE + S * S;

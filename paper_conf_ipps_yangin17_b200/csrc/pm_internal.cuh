@@ -15,6 +15,16 @@ namespace pm {
 extern std::atomic<int64_t> g_launches;
 inline void note_launch(int64_t n = 1) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
+// Stream-ordered scratch from a library-owned memory pool per device whose
+// release threshold is unlimited: after the first call, scratch allocations
+// are served from the pool without re-mapping memory (the default pool
+// returns memory to the driver at every synchronisation, ~1 ms per call).
+cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st);
+template <typename T>
+inline cudaError_t scratch_alloc(T** p, size_t bytes, cudaStream_t st) {
+  return scratch_alloc(reinterpret_cast<void**>(p), bytes, st);
+}
+
 #define PM_CUDA_TRY(expr)                         \
   do {                                            \
     cudaError_t _e = (expr);                      \

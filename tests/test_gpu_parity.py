@@ -156,7 +156,7 @@ def test_local_search_parity_config2(method, fam):
     _check_ls(oracle_E(fam, 512, 16), method)
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "cta", "class"])
 def test_local_search_parity_config3(method):
     ref = _check_ls(oracle_E("smooth", 1024, 16), method)
     assert ref[1] >= 3
@@ -309,13 +309,20 @@ def test_launch_count_increments():
     assert pm.launch_count() - n0 >= 5   # 2 pack + E + iota + search + cost
 
 
-@pytest.mark.parametrize("N,M", [(1600, 40), (1150, 25), (1344, 24), (2048, 32)])
+@pytest.mark.parametrize("N,M", [(1600, 40), (1152, 32), (1440, 32)])
 def test_local_search_window_sizes(N, M):
-    # S = 1600 and 2116 (K = 16 window), 3136 and 4096 (K = 8 window), grayscale noise
+    # S = 1600, 1296, 2025 (the K = 4 window tier, S in (1024, 2048]), grayscale noise
     _check_ls(oracle_E("noise", N, M, 1), "window")
 
 
-@pytest.mark.parametrize("S_side", [33, 45, 63])
+@pytest.mark.parametrize("S_side", [31, 33, 45])
 def test_local_search_window_odd_mid(S_side):
-    # odd S between the window tiers (1089, 2025, 3969)
+    # odd S around the window tiers (961, 1089, 2025)
     _check_ls(oracle_E("smooth", S_side * 4, 4, 3), "window")
+
+
+def test_local_search_window_rejects_large_S():
+    E = torch.zeros((2116, 2116), dtype=torch.int32, device=DEV)
+    with pytest.raises(pm.PMError) as ei:
+        pm.local_search(E, method="window")
+    assert ei.value.status == pm.PM_ERR_UNSUPPORTED
