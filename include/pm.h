@@ -99,7 +99,7 @@ int32_t pm_num_colors(int32_t S);
 /* Edge groups P_{class_begin+1} .. P_{class_end}, 0-indexed slots,
  * in the paper's group order and, inside a group, by increasing smaller index
  * (exactly the printed K_16 table for S = 16).  Host-side, for tests and
- * inspection; the kernels generate the same groups on the fly (reading R7:
+ * inspection; the kernels generate the same groups on the fly (reading R8:
  * pairs u + v == 2i + 1 (mod m), m = S-1 for even S, m = S for odd S; the
  * fixed point joins vertex S when S is even and idles when S is odd).
  *   h_pairs : int32 [class_end - class_begin][S/2][2], each (u, v) with u < v;

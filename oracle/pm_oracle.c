@@ -84,7 +84,7 @@ int32_t or_num_colors(int32_t S) {
   return (S % 2 == 0) ? S - 1 : S;
 }
 
-/* Edge groups P_1..P_m, 0-indexed slots.  Reading R7 (the round-
+/* Edge groups P_1..P_m, 0-indexed slots.  Reading R8 (the round-
  * robin 1-factorisation that reproduces the printed K_16 groups exactly):
  * with m = S-1 (S even) or m = S (S odd) and 1-indexed vertices,
  *   P_i = {(u, v) : 1 <= u < v <= m, u + v == 2i + 1 (mod m)}

@@ -33,7 +33,7 @@ inline cudaError_t scratch_alloc(T** p, size_t bytes, cudaStream_t st) {
 
 // ----------------------------------------------------------------------------
 // Colour classes of K_S (Theorem 1; groups P:152-203), generated on the
-// fly.  0-indexed slots, class c in [0, ncls).  Reading R7: with m = S-1 (S
+// fly.  0-indexed slots, class c in [0, ncls).  Reading R8: with m = S-1 (S
 // even) or m = S (S odd), class c pairs slots whose sum is 2c+1 (mod m); its
 // fixed point u0 = (c + (m+1)/2) mod m (the solution of 2u0 == 2c+1) is joined
 // to slot S-1 when S is even and idles when S is odd.  Enumerated here as
