@@ -128,7 +128,8 @@ pm_status_t pm_local_search(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t
                             pm_stream_t stream);
 
 /* pm_local_search with an explicit method (pm_ls_method_t) and an optional
- * per-round swap log h_swaps_per_round[0 .. min(rounds, len)-1] (may be NULL). */
+ * per-round swap log h_swaps_per_round[0 .. min(rounds, len)-1] (may be NULL;
+ * entries from index `rounds` on are written as zero, up to len). */
 pm_status_t pm_local_search_ex(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
                                int32_t max_rounds, int32_t method,
                                int32_t* h_rounds, int64_t* h_swaps,

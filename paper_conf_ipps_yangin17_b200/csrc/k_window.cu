@@ -65,24 +65,25 @@ template <int K>
 struct WinSmem {
   static constexpr int KS = K + 4;   // stored entries per slot: an aligned superset of K
   static size_t bytes(int32_t S) {
-    return sizeof(int32_t) * ((size_t)S * 7 + (size_t)2 * KS * win_stride(S) + 64);
+    return sizeof(int32_t) * ((size_t)S * 8 + (size_t)2 * KS * win_stride(S) + 64);
   }
 };
 
 // Per regular slot x, two windows in shared memory, stored transposed
 // (entry-major, stride SP == 1 mod 32: the slots of one class are read
 // conflict-free).  Each holds a 16-byte-aligned superset of K entries of a
-// sigma-permuted row, loaded with unconditional LDG.128 / 4 x STS; off[x] is
-// the offset of the first wanted entry inside the superset:
-//   W [off[x] + j][x] = E[r[x]][p_{wb+j}(x)]  = Ep[r[x]][sigma(1-x) + wb + j]   (class window)
-//   SW[swoff[x] + i][x] = E[r[x]][x + 2(i+1)] = Ep[r[x]][sigma(x) + i + 1]      (diagonal window)
+// sigma-permuted row, loaded with unconditional LDG.128 / 4 x STS; woff[x]
+// (kept next to d[x]) / swoff[x] = (sigma(x)+1) & 3 locate the first wanted
+// entry inside the superset:
+//   W [woff[x] + j][x]  = E[r[x]][p_{wb+j}(x)]  = Ep[r[x]][sigma(1-x) + wb + j]  (class window)
+//   SW[swoff[x] + i][x] = E[r[x]][x + 2(i+1)]   = Ep[r[x]][sigma(x) + i + 1]     (diagonal window)
 // Swap of regular slots (u, v) in class c = wb + j, a = r[u], b = r[v]: since
 // p_{c+i}(u) = v + 2i and p_{c+i}(v) = u + 2i,
 //   W'[j+i][u] = E[b][v+2i] = SW[i-1][v]     SW'[i-1][u] = E[b][u+2i] = W[j+i][v]
 // (and symmetrically for v): the swap is an exchange of shared-memory entries
-// with no global access.  SW' entries beyond the window are stale and are
-// reloaded at the next window (slots swapped during window w are those with
-// dgen == w) but never read before: a later swap at class c'' > c needs
+// with no global access.  SW' entries beyond the window are stale; the slot is
+// put on the dirty list of its window and its SW is reloaded at the next
+// window, and they are never read before: a later swap at class c'' > c needs
 // offsets < jmax - (c'' - wb).  SW does not depend on the class, so clean
 // slots keep theirs across windows and rounds.  Slot L = S-1 walks the plain
 // row E[r[L]][u0(c)] (u0(c) = c + (m+1)/2 advances by one per class); the rare
@@ -96,15 +97,15 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
   constexpr int NP = KS / 4;       // 16-byte pieces per window
   extern __shared__ __align__(16) int32_t sm[];
   const int32_t SP = win_stride(S);
-  int2* s_do = reinterpret_cast<int2*>(sm);   // {d[x] = E[r[x]][x], off[x]}
+  int2* s_do = reinterpret_cast<int2*>(sm);   // {d[x] = E[r[x]][x], woff[x]}
   int32_t* s_r = sm + 2 * S;       // r[x]: tile at slot x
   int32_t* s_last = s_r + S;       // E[t][L] per tile t (even S)
   int32_t* s_sig = s_last + S;     // sigma(x)
-  int32_t* s_swoff = s_sig + S;    // offset of SW inside its superset
-  int32_t* s_dgen = s_swoff + S;   // window id of x's last swap (SW reload at the next window)
-  int32_t* s_W = s_dgen + S;       // [KS][SP]
+  int32_t* s_src = s_sig + S;      // element offset of x's W superset in Ep (current window)
+  int32_t* s_dgen = s_src + S;     // window id of x's last swap (its SW is reloaded at the next window)
+  int32_t* s_W = s_dgen + 2 * S;   // [KS][SP]
   int32_t* s_SW = s_W + (size_t)KS * SP;     // [KS][SP]
-  int32_t* s_ctl = s_SW + (size_t)KS * SP;   // [0..2] first-fire slots, [8..40] reduction
+  int32_t* s_ctl = s_SW + (size_t)KS * SP;   // [0..2] first-fire, [4..5] dirty counts, [8..40] reduction
   const Classes cl(S);
   const int32_t m = cl.m, H = cl.half;
   const bool even = (S % 2) == 0;
@@ -133,12 +134,10 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
   for (int32_t x = tid; x < S; x += T) {
     s_do[x] = make_int2(__ldg(E + (int64_t)s_r[x] * ld + x), 0);
     if (even) s_last[x] = __ldg(E + (int64_t)x * ld + L);
-    const int32_t sg = (x < m) ? (int32_t)(((int64_t)x * H) % m) : 0;
-    s_sig[x] = sg;
-    s_swoff[x] = (sg + 1) & 3;
-    s_dgen[x] = -1;                   // window 0 loads every SW
+    s_sig[x] = (x < m) ? (int32_t)(((int64_t)x * H) % m) : 0;
+    s_dgen[x] = -1;
   }
-  if (tid < 3) s_ctl[tid] = INT32_MAX;
+  if (tid < 8) s_ctl[tid] = (tid < 3) ? INT32_MAX : 0;
   __syncthreads();
 
   auto wrap = [&](int32_t q) -> int32_t {   // q in (-m, 2m)
@@ -146,56 +145,50 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     if (q >= m) q -= m;
     return q;
   };
-  // window `wid` for classes [wb, wb + jmax): W of every slot, SW of slots
-  // swapped during window wid - 1 (and all at wid = 0)
-  auto fill = [&](int32_t wb, int32_t jmax, int32_t wid) {
-    constexpr int U = MAXT <= 512 ? 4 : 2;   // loads in flight per thread
+  // Window w for classes [wb, wb + jmax): W of every slot; SW of the slots
+  // swapped during window w-1 (every slot at w = 0 or after a list overflow).
+  auto fill = [&](int32_t wb, int32_t jmax, int32_t w) {
+    constexpr int U = MAXT <= 512 ? 4 : 2;   // 16-byte loads in flight per thread
     __syncthreads();
-    const int32_t total = nreg * NP;
-    for (int32_t f0 = 0; f0 < total; f0 += U * T) {
+    for (int32_t x = tid; x < nreg; x += T) {
+      const int32_t pos = wrap(wb + H - s_sig[x]);
+      const int32_t base = pos & ~3;
+      s_src[x] = s_r[x] * (int32_t)ldp + base;
+      s_do[x].y = (pos - base) | (((s_sig[x] + 1) & 3) << 2);   // woff | swoff << 2
+    }
+    __syncthreads();
+    const int32_t totW = nreg * NP;
+    for (int32_t f0 = 0; f0 < totW; f0 += U * T) {
       int4 val[U];
-      int32_t dst[U];
 #pragma unroll
       for (int uu = 0; uu < U; ++uu) {
         const int32_t f = f0 + uu * T + tid;
-        dst[uu] = -1;
-        if (f < total) {
+        if (f < totW) {
           const int32_t x = f / NP, q = f - x * NP;
-          const int32_t pos = wrap(wb + H - s_sig[x]);
-          const int32_t base = pos & ~3;
-          val[uu] = __ldg(reinterpret_cast<const int4*>(Ep + (int64_t)s_r[x] * ldp + base) + q);
-          if (q == 0) s_do[x].y = pos - base;
-          dst[uu] = (4 * q) * SP + x;
+          val[uu] = __ldg(reinterpret_cast<const int4*>(Ep + s_src[x]) + q);
         }
       }
 #pragma unroll
       for (int uu = 0; uu < U; ++uu) {
-        if (dst[uu] < 0) continue;
-        int32_t* w = s_W + dst[uu];
-        w[0] = val[uu].x; w[SP] = val[uu].y; w[2 * SP] = val[uu].z; w[3 * SP] = val[uu].w;
+        const int32_t f = f0 + uu * T + tid;
+        if (f < totW) {
+          const int32_t x = f / NP, q = f - x * NP;
+          int32_t* d = s_W + (4 * q) * SP + x;
+          d[0] = val[uu].x; d[SP] = val[uu].y; d[2 * SP] = val[uu].z; d[3 * SP] = val[uu].w;
+        }
       }
     }
-    for (int32_t f0 = 0; f0 < total; f0 += U * T) {
-      int4 val[U];
-      int32_t dst[U];
+    // SW of slots swapped during window w-1 (all slots at w = 0): one thread per slot
+    for (int32_t x = tid; x < nreg; x += T) {
+      if (w != 0 && s_dgen[x] != w - 1) continue;
+      const int4* src = reinterpret_cast<const int4*>(Ep + s_r[x] * (int32_t)ldp + ((s_sig[x] + 1) & ~3));
+      int4 val[NP];
 #pragma unroll
-      for (int uu = 0; uu < U; ++uu) {
-        const int32_t f = f0 + uu * T + tid;
-        dst[uu] = -1;
-        if (f < total) {
-          const int32_t x = f / NP, q = f - x * NP;
-          if (s_dgen[x] == wid - 1) {
-            const int32_t base = (s_sig[x] + 1) & ~3;
-            val[uu] = __ldg(reinterpret_cast<const int4*>(Ep + (int64_t)s_r[x] * ldp + base) + q);
-            dst[uu] = (4 * q) * SP + x;
-          }
-        }
-      }
+      for (int q = 0; q < NP; ++q) val[q] = __ldg(src + q);
 #pragma unroll
-      for (int uu = 0; uu < U; ++uu) {
-        if (dst[uu] < 0) continue;
-        int32_t* w = s_SW + dst[uu];
-        w[0] = val[uu].x; w[SP] = val[uu].y; w[2 * SP] = val[uu].z; w[3 * SP] = val[uu].w;
+      for (int q = 0; q < NP; ++q) {
+        int32_t* d = s_SW + (4 * q) * SP + x;
+        d[0] = val[q].x; d[SP] = val[q].y; d[2 * SP] = val[q].z; d[3 * SP] = val[q].w;
       }
     }
     if (even) {
@@ -214,7 +207,7 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
       if (k < cl.npairs) cl.pair(c, k, pu[q], pv[q]);
     }
   };
-  auto advance = [&](int32_t delta) {   // classes are consecutive: u0 + k, u0 - k, u0 all shift by +1
+  auto advance = [&](int32_t delta) {   // consecutive classes: u0 + k, u0 - k, u0 all shift by +1
 #pragma unroll
     for (int q = 0; q < PPT; ++q) {
       const int32_t k = tid + q * T;
@@ -224,13 +217,11 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     }
   };
   // O(u), O(v) at window offset j; fire iff d[u] + d[v] > O(u) + O(v)
-  auto eval = [&](int q, int32_t u, int32_t v, int32_t j, int2& du, int2& dv, int32_t& ou, int32_t& ov) -> bool {
-    const int32_t k = tid + q * T;
-    du = s_do[u];
-    dv = s_do[v];
-    if (even && k == 0) ou = s_last[s_r[u]];          // u = u0(c), partner L
-    else ou = s_W[(j + du.y) * SP + u];
-    ov = s_W[(j + dv.y) * SP + v];
+  auto eval = [&](bool special, int32_t u, int32_t v, int32_t j, int32_t& ou, int32_t& ov) -> bool {
+    const int2 du = s_do[u];
+    const int2 dv = s_do[v];
+    ou = special ? s_last[s_r[u]] : s_W[(j + (du.y & 3)) * SP + u];   // special: u = u0(c), partner L
+    ov = s_W[(j + (dv.y & 3)) * SP + v];
     return (int64_t)du.x + dv.x > (int64_t)ou + ov;
   };
 
@@ -238,7 +229,14 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
   int64_t total = 0;
   int status = PM_OK;
   uint32_t batch = 0;
-  int32_t wid = 0;
+  int32_t wid = -1;
+#ifdef PM_LS_PROFILE
+  long long t_round = clock64();
+  int32_t n_apply = 0, n_spec = 0;
+  long long t_fill = 0, t_spec = 0, t_apply = 0;
+  long long t_ph[3] = {0, 0, 0};
+  long long tA = 0, tB = 0;
+#endif
   int32_t B = 1;
   for (;;) {                                           // Alg. 2 line 1
     int mysw = 0;
@@ -248,8 +246,14 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     while (c < cl.ncls) {                              // line 3, classes in order
       if (c >= wb + K) {
         wb = c;
-        fill(wb, min(K, cl.ncls - wb), wid);
         ++wid;
+#ifdef PM_LS_PROFILE
+        const long long tf0 = clock64();
+#endif
+        fill(wb, min(K, cl.ncls - wb), wid);
+#ifdef PM_LS_PROFILE
+        t_fill += clock64() - tf0;
+#endif
       }
       const int32_t jmax = min(K, cl.ncls - wb);
       int32_t* first_slot = s_ctl + (batch % 3);
@@ -257,24 +261,51 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
       ++batch;
       const int32_t cend = min(c + B, wb + jmax);
       int32_t cc = c;
+#ifdef PM_LS_PROFILE
+      const long long ts0 = clock64();
+#endif
       if (cend - c > 1) {
         // speculative: all pairs of classes [c, cend) on the current state
         const int32_t nb = cend - c;
 #pragma unroll
         for (int q = 0; q < PPT; ++q) {
-          if (tid + q * T >= cl.npairs) continue;
+          const int32_t k = tid + q * T;
+          if (k >= cl.npairs) continue;
+          const bool special = even && k == 0;
           int32_t u = pu[q], v = pv[q];
-          const bool special = even && tid + q * T == 0;
-          for (int32_t jj = 0; jj < nb; ++jj) {
-            int2 du, dv;
-            int32_t ou, ov;
-            if (eval(q, u, v, c + jj - wb, du, dv, ou, ov)) { atomicMin(first_slot, jj); break; }
-            u = (u + 1 == m) ? 0 : u + 1;
-            if (!special) v = (v + 1 == m) ? 0 : v + 1;
+          // 4 classes per step: all shared-memory loads issued before any test
+          for (int32_t jj0 = 0; jj0 < nb; jj0 += 4) {
+            int32_t us[4], vs[4];
+            int2 du[4], dv[4];
+            int32_t ou[4], ov[4];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+              us[t] = u; vs[t] = v;
+              u = (u + 1 == m) ? 0 : u + 1;
+              if (!special) v = (v + 1 == m) ? 0 : v + 1;
+            }
+#pragma unroll
+            for (int t = 0; t < 4; ++t) { du[t] = s_do[us[t]]; dv[t] = s_do[vs[t]]; }
+            const int32_t j0 = c + jj0 - wb;
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+              // entries past the window end are read but never used (j < KS always)
+              ou[t] = special ? s_last[s_r[us[t]]] : s_W[(j0 + t + (du[t].y & 3)) * SP + us[t]];
+              ov[t] = s_W[(j0 + t + (dv[t].y & 3)) * SP + vs[t]];
+            }
+            int hit = -1;
+#pragma unroll
+            for (int t = 3; t >= 0; --t)
+              if (jj0 + t < nb && (int64_t)du[t].x + dv[t].x > (int64_t)ou[t] + ov[t]) hit = t;
+            if (hit >= 0) { atomicMin(first_slot, jj0 + hit); break; }
           }
         }
         __syncthreads();
         const int32_t first = *first_slot;
+#ifdef PM_LS_PROFILE
+        ++n_spec;
+        t_spec += clock64() - ts0;
+#endif
         if (first == INT32_MAX) {
           advance(nb);
           c = cend;
@@ -292,28 +323,38 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
       for (int q = 0; q < PPT; ++q) {                  // warp-uniform
         const int32_t k = tid + q * T;
         const int32_t u = pu[q], v = pv[q];
-        int32_t a = 0, b = 0;
-        int2 du, dv;
-        int32_t ou = 0, ov = 0;
+        const bool special = even && k == 0;
+        int32_t a = 0, b = 0, yu = 0, yv = 0;
         bool f = false;
-        if (k < cl.npairs && eval(q, u, v, j, du, dv, ou, ov)) {
-          a = s_r[u]; b = s_r[v];
-          s_r[u] = b; s_r[v] = a;
-          s_do[u].x = ov; s_do[v].x = ou;  // d[u] = E[b][u] = O(v), d[v] = E[a][v] = O(u)
-          s_dgen[u] = wid - 1; s_dgen[v] = wid - 1;
-          ++mysw;
-          fired = 1;
-          f = true;
+        if (k < cl.npairs) {
+          const int2 du = s_do[u];
+          const int2 dv = s_do[v];
+          yu = du.y; yv = dv.y;
+          const int32_t ou = special ? s_last[s_r[u]] : s_W[(j + (yu & 3)) * SP + u];
+          const int32_t ov = s_W[(j + (yv & 3)) * SP + v];
+          if ((int64_t)du.x + dv.x > (int64_t)ou + ov) {
+            a = s_r[u]; b = s_r[v];
+            s_r[u] = b; s_r[v] = a;
+            s_do[u].x = ov; s_do[v].x = ou;  // d[u] = E[b][u] = O(v), d[v] = E[a][v] = O(u)
+            s_dgen[u] = wid; s_dgen[v] = wid;
+            ++mysw;
+            fired = 1;
+            f = true;
+          }
         }
+#ifdef PM_LS_PROFILE
+        tA = clock64();
+#endif
         unsigned mask = __ballot_sync(0xffffffffu, f);
         while (mask) {
           const int sl = __ffs(mask) - 1;
           mask &= mask - 1;
           const int32_t su = __shfl_sync(0xffffffffu, u, sl), sv = __shfl_sync(0xffffffffu, v, sl);
-          const bool sfixed = even && (__shfl_sync(0xffffffffu, k, sl) == 0);
-          const int32_t ofu = s_do[su].y, ofv = s_do[sv].y;
+          const int32_t syu = __shfl_sync(0xffffffffu, yu, sl), syv = __shfl_sync(0xffffffffu, yv, sl);
+          const bool sfixed = __shfl_sync(0xffffffffu, special, sl);
+          const int32_t ofu = syu & 3, ofv = syv & 3;
           if (!sfixed) {
-            const int32_t swu = s_swoff[su], swv = s_swoff[sv];
+            const int32_t swu = syu >> 2, swv = syv >> 2;
             for (int32_t jj = j + 1 + lane; jj < jmax; jj += 32) {
               const int32_t i = jj - j - 1;
               int32_t* Wu = s_W + (jj + ofu) * SP + su;
@@ -328,7 +369,7 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
             // (u0, L): u0 now holds b (walks Ep[b][sigma(u0) + i]), L holds a
             // (walks E[a][u0 + i]); reload from global (rare: 1 pair per class)
             const int32_t sa = __shfl_sync(0xffffffffu, a, sl), sb = __shfl_sync(0xffffffffu, b, sl);
-            const int32_t sg = s_sig[su], swu = s_swoff[su];
+            const int32_t sg = s_sig[su], swu = syu >> 2;
             for (int32_t jj = j + 1 + lane; jj < jmax; jj += 32) {
               const int32_t i = jj - j;
               const int32_t e1 = __ldg(Ep + (int64_t)sb * ldp + sg + i);
@@ -340,7 +381,16 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
           }
         }
       }
+#ifdef PM_LS_PROFILE
+      tB = clock64();
+#endif
       const int any = __syncthreads_or(fired);
+#ifdef PM_LS_PROFILE
+      ++n_apply;
+      const long long tC = clock64();
+      t_apply += tC - ts0;
+      t_ph[0] += tA - ts0; t_ph[1] += tB - tA; t_ph[2] += tC - tB;
+#endif
       if (cend - c <= 1 && !any) B = 2;                 // quiet class: start speculating
       advance(1);
       c = cc + 1;
@@ -356,6 +406,31 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     int rs = 0;
     for (int w = 0; w < (T >> 5); ++w) rs += red[w];
     if (tid == 0 && rounds < max_log) per_round[rounds] = rs;
+#ifdef PM_LS_PROFILE
+    if (tid == 0 && max_log >= 1024 && rounds < 128) {
+      const long long now = clock64();
+      per_round[512 + rounds] = now - t_round;
+      per_round[640 + rounds] = n_apply;
+      per_round[768 + rounds] = n_spec;
+      per_round[896 + rounds] = t_fill;
+      per_round[896 + 32 + rounds] = t_spec;
+      per_round[896 + 64 + rounds] = t_apply;
+      t_round = now;
+    }
+    if (tid == 32 && max_log >= 1024 && rounds < 16) {
+      per_round[256 + rounds] = t_ph[0];
+      per_round[256 + 16 + rounds] = t_ph[1];
+      per_round[256 + 32 + rounds] = t_ph[2];
+    }
+    if (tid == 0 && max_log >= 1024 && rounds < 16) {
+      per_round[320 + rounds] = t_ph[0];
+      per_round[320 + 16 + rounds] = t_ph[1];
+      per_round[320 + 32 + rounds] = t_ph[2];
+    }
+    t_ph[0] = t_ph[1] = t_ph[2] = 0;
+    n_apply = n_spec = 0;
+    t_fill = t_spec = t_apply = 0;
+#endif
     rounds += 1;
     total += rs;
     if (rs == 0) break;

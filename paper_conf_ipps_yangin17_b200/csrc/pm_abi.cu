@@ -92,10 +92,8 @@ pm_status_t local_search_impl(const int32_t* d_E, int64_t ld_E, int32_t S, int32
   if (used == PM_LS_CLASS) note_launch(hres.rounds * ls_class_launches_per_round(S));
   if (h_rounds) *h_rounds = (int32_t)hres.rounds;
   if (h_swaps) *h_swaps = hres.swaps;
-  if (h_per_round && len > 0) {
-    const int32_t n = (int32_t)std::min<int64_t>(hres.rounds, (int64_t)hlog.size());
-    for (int32_t i = 0; i < n; ++i) h_per_round[i] = hlog[i];
-  }
+  if (h_per_round && len > 0)   // entries at and beyond `rounds` are zero
+    for (size_t i = 0; i < hlog.size(); ++i) h_per_round[i] = hlog[i];
   return (pm_status_t)hres.status;
 }
 
