@@ -145,6 +145,9 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
                                   int32_t max_rounds, int32_t method, int64_t* d_result,
                                   pm_stream_t stream);
 
+/* The method PM_LS_AUTO selects for S on the current device (host-only). */
+int32_t pm_ls_auto_method(int32_t S);
+
 /* Largest S the single-CTA methods accept on this device (shared-memory
  * bound); 0 if no device. */
 int32_t pm_ls_cta_max_S(void);

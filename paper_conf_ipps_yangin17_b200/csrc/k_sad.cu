@@ -87,12 +87,35 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
 
-// A: input tiles, rows [0, nrows) (already offset by row_begin); B: target
-// tiles, rows [0, S).  kw_split: K words handled by one blockIdx.z slice.
-template <bool kAtomic>
+// Where the K bytes of a tile live.  Packed: tile t at A + t*ldt (bytes
+// contiguous).  Image (Step 1 fused into the loader, used when a tile row is a
+// whole number of 16-byte pieces): tile t = grid cell (t / g, t % g) of a u8
+// HWC image; its 16-byte piece p is row y = p / R (R = M*C/16 pieces per tile
+// row) at byte offset (p % R)*16 of that row, i.e. the same (y, x, c) byte
+// order as k_pack produces.
+struct SadGeom {
+  const uint8_t* A;        // input tiles (packed, already offset by row_begin) or input image
+  const uint8_t* B;        // target tiles or target image
+  int64_t ldt;             // packed: tile stride in bytes
+  int64_t rowbytes;        // image: N*C
+  int32_t a_tile0;         // image: tile index of local row 0 (row_begin)
+  int32_t g, M, R, MC;     // image: tiles per grid row, tile side, pieces per tile row, M*C
+};
+
+template <bool kImage>
+__device__ __forceinline__ const uint8_t* sad_tile_base(const SadGeom& geo, const uint8_t* img, int32_t t) {
+  if (kImage) {
+    const int32_t ty = t / geo.g, tx = t - ty * geo.g;
+    return img + (int64_t)ty * geo.M * geo.rowbytes + (int64_t)tx * geo.MC;
+  }
+  return img + (int64_t)t * geo.ldt;
+}
+
+// nrows rows of A (input tiles), S columns (target tiles).  kw_split: K words
+// handled by one blockIdx.z slice.
+template <bool kAtomic, bool kImage>
 __global__ void __launch_bounds__(sad::kThreads, 1)
-k_sad(const uint8_t* __restrict__ A, const uint8_t* __restrict__ B, int64_t ldt, int32_t nrows,
-      int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE) {
+k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE) {
   using namespace sad;
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t* sA = smem;                                 // [kStages][BM][ROWW]
@@ -101,13 +124,14 @@ k_sad(const uint8_t* __restrict__ A, const uint8_t* __restrict__ B, int64_t ldt,
   const int tid = threadIdx.x;
   const int tx = tid & 15, ty = tid >> 4;
   const int32_t row0 = blockIdx.y * BM, col0 = blockIdx.x * BN;
-  const int64_t kbyte0 = (int64_t)blockIdx.z * kw_split * 4;
+  const int32_t piece0 = blockIdx.z * kw_split / 4;    // first 16-byte piece of this K slice
   const int nkb = kw_split / BKW;
 
-  // Loader: per operand and stage, BM rows x 64 B = 512 16-byte chunks; thread
-  // tid copies chunks q = tid and q = tid + 256 (row q >> 2, part q & 3).
-  const uint8_t* srcA[2];
-  const uint8_t* srcB[2];
+  // Loader: per operand and stage, BM rows x 64 B = 512 16-byte pieces; thread
+  // tid copies pieces q = tid and q = tid + 256 (row q >> 2, part q & 3).
+  const uint8_t* baseA[2];
+  const uint8_t* baseB[2];
+  int part4[2];
   int dst_off[2];
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
@@ -115,15 +139,24 @@ k_sad(const uint8_t* __restrict__ A, const uint8_t* __restrict__ B, int64_t ldt,
     const int r = q >> 2, part = q & 3;
     int32_t ra = row0 + r; if (ra >= nrows) ra = nrows - 1;   // clamp: loaded, never stored
     int32_t rb = col0 + r; if (rb >= S) rb = S - 1;
-    srcA[h] = A + (int64_t)ra * ldt + kbyte0 + part * 16;
-    srcB[h] = B + (int64_t)rb * ldt + kbyte0 + part * 16;
+    baseA[h] = sad_tile_base<kImage>(geo, geo.A, kImage ? geo.a_tile0 + ra : ra);
+    baseB[h] = sad_tile_base<kImage>(geo, geo.B, rb);
+    part4[h] = part;
     dst_off[h] = r * ROWW + part * 4;
   }
   auto load_stage = [&](int kb, int stage) {
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-      cp_async16(sA + stage * BM * ROWW + dst_off[h], srcA[h] + kb * (BKW * 4));
-      cp_async16(sB + stage * BN * ROWW + dst_off[h], srcB[h] + kb * (BKW * 4));
+      const int32_t p = piece0 + kb * (BKW / 4) + part4[h];
+      int64_t off;
+      if (kImage) {
+        const int32_t y = p / geo.R;
+        off = (int64_t)y * geo.rowbytes + (p - y * geo.R) * 16;
+      } else {
+        off = (int64_t)p * 16;
+      }
+      cp_async16(sA + stage * BM * ROWW + dst_off[h], baseA[h] + off);
+      cp_async16(sB + stage * BN * ROWW + dst_off[h], baseB[h] + off);
     }
   };
 
@@ -204,23 +237,28 @@ static int choose_split(int64_t tiles, int nkb, int sms) {
   return best;
 }
 
-cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
-                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st) {
+template <bool kAtomic, bool kImage>
+static cudaError_t sad_set_attr() {
+  return cudaFuncSetAttribute(k_sad<kAtomic, kImage>, cudaFuncAttributeMaxDynamicSharedMemorySize, sad::kSmemBytes);
+}
+
+static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows, int32_t S, int32_t P,
+                                   int32_t* E, int64_t ldE, cudaStream_t st) {
   using namespace sad;
-  (void)P;
   if (nrows <= 0 || S <= 0) return cudaSuccess;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   static std::atomic<uint64_t> attr_done{0};   // one bit per device ordinal
   if (dev < 64 && !(attr_done.load() & (1ull << dev))) {
-    cudaError_t e = cudaFuncSetAttribute(k_sad<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(k_sad<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBytes);
-    if (e != cudaSuccess) return e;
+    cudaError_t e;
+    if ((e = sad_set_attr<false, false>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<true, false>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<false, true>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<true, true>()) != cudaSuccess) return e;
     attr_done.fetch_or(1ull << dev);
   }
-  const int kw = (int)(ldt / 4);
+  const int kw = image ? P / 4 : (int)(geo.ldt / 4);
   const int nkb = kw / BKW;
   const int64_t gx = (S + BN - 1) / BN, gy = (nrows + BM - 1) / BM;
   if (gy > 65535) return cudaErrorInvalidValue;
@@ -232,12 +270,38 @@ cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t 
         ? cudaMemsetAsync(E, 0, sizeof(int32_t) * (size_t)nrows * S, st)
         : cudaMemset2DAsync(E, sizeof(int32_t) * ldE, 0, sizeof(int32_t) * S, nrows, st);
     if (e != cudaSuccess) return e;
-    k_sad<true><<<grid, kThreads, kSmemBytes, st>>>(A, B, ldt, nrows, S, kw / split, E, ldE);
+    if (image) k_sad<true, true><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw / split, E, ldE);
+    else k_sad<true, false><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw / split, E, ldE);
   } else {
-    k_sad<false><<<grid, kThreads, kSmemBytes, st>>>(A, B, ldt, nrows, S, kw, E, ldE);
+    if (image) k_sad<false, true><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw, E, ldE);
+    else k_sad<false, false><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw, E, ldE);
   }
   note_launch();
   return cudaGetLastError();
+}
+
+cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
+                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st) {
+  SadGeom geo = {};
+  geo.A = A; geo.B = B; geo.ldt = ldt;
+  return launch_sad_geom(geo, false, nrows, S, P, E, ldE, st);
+}
+
+bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C) {
+  const int64_t MC = (int64_t)M * C, P = MC * M;
+  return MC % 16 == 0 && P % 64 == 0 && ((int64_t)N * C) % 16 == 0 &&
+         (reinterpret_cast<uintptr_t>(I) % 16) == 0 && (reinterpret_cast<uintptr_t>(T) % 16) == 0;
+}
+
+cudaError_t launch_sad_image(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C,
+                             int32_t row_begin, int32_t row_end, int32_t* E, int64_t ldE, cudaStream_t st) {
+  SadGeom geo = {};
+  geo.A = I; geo.B = T;
+  geo.rowbytes = (int64_t)N * C;
+  geo.a_tile0 = row_begin;
+  geo.g = N / M; geo.M = M; geo.MC = M * C; geo.R = M * C / 16;
+  const int32_t S = geo.g * geo.g;
+  return launch_sad_geom(geo, true, row_end - row_begin, S, M * M * C, E, ldE, st);
 }
 
 }  // namespace pm

@@ -294,8 +294,7 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
                              int32_t method, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                              cudaStream_t st, int32_t* used_method) {
   const int32_t cta_max = ls_cta_max_S();
-  if (method == PM_LS_AUTO)
-    method = (S <= ls_window_max_S()) ? PM_LS_WINDOW : (S <= cta_max) ? PM_LS_CTA : PM_LS_CLASS;
+  if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
   if (used_method) *used_method = method;
   switch (method) {
     case PM_LS_CLASS:

@@ -151,6 +151,13 @@ pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target, int
   if (row_begin == row_end) return PM_OK;   // empty shard: nothing to do, pointers unused
   if (!d_input || !d_target || !d_E) return PM_ERR_INVALID;
   cudaStream_t st = (cudaStream_t)stream;
+  // Step 1 fused into the E loader where the two pack launches would cost more
+  // than the loader's per-stage address arithmetic (measured: fused ~8 % slower
+  // per pair at S >= 16384, pack overhead dominant at S <= 4096).
+  if (S <= 4096 && sad_image_ok(d_input, d_target, N, M, C)) {
+    PM_CUDA_TRY(launch_sad_image(d_input, d_target, N, M, C, row_begin, row_end, d_E, ld_E, st));
+    return PM_OK;
+  }
   const int64_t ldt = pm_tile_stride(M, C);
   const int32_t nrows = row_end - row_begin;
   DevBuf buf;
@@ -212,6 +219,10 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
 }
 
 int32_t pm_ls_cta_max_S(void) { return ls_cta_max_S(); }
+
+int32_t pm_ls_auto_method(int32_t S) {
+  return (S <= ls_window_max_S()) ? PM_LS_WINDOW : (S <= ls_cta_max_S()) ? PM_LS_CTA : PM_LS_CLASS;
+}
 
 pm_status_t pm_cost_async(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int64_t* d_cost,
                           pm_stream_t stream) {

@@ -84,6 +84,11 @@ cudaError_t launch_pack(const uint8_t* img, int32_t N, int32_t M, int32_t C, uin
                         int64_t ld_tiles, int32_t tile_begin, int32_t tile_end, cudaStream_t st);
 cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
                        int32_t P, int32_t* E, int64_t ldE, cudaStream_t st);
+// Step 1 fused into the E kernel's loader (no packed tiles): requires
+// sad_image_ok (a tile row is a whole number of 16-byte pieces, P % 64 == 0).
+bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C);
+cudaError_t launch_sad_image(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C,
+                             int32_t row_begin, int32_t row_end, int32_t* E, int64_t ldE, cudaStream_t st);
 
 // Device-side result of one search; layout = the int64 [3] of
 // pm_local_search_async's d_result: {status, rounds, swaps}.

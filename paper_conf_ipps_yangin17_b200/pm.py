@@ -39,6 +39,7 @@ _SIGS = [
     ("pm_local_search_ex", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P, _I32, _P]),
     ("pm_local_search_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P]),
     ("pm_ls_cta_max_S", _I32, []),
+    ("pm_ls_auto_method", _I32, [_I32]),
     ("pm_init_identity", ctypes.c_int, [_P, _I32, _P]),
     ("pm_cost", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P]),
     ("pm_cost_async", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P]),
@@ -207,6 +208,12 @@ def local_search_async(E, perm, result, max_rounds: int = 0, method: str = "auto
 
 def ls_cta_max_S() -> int:
     return int(lib().pm_ls_cta_max_S())
+
+
+def ls_auto_method(S: int) -> str:
+    """Name of the method PM_LS_AUTO picks for S on the current device."""
+    code = int(lib().pm_ls_auto_method(S))
+    return {v: k for k, v in METHODS.items()}[code]
 
 
 def init_identity(perm, stream=None):

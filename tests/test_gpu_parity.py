@@ -326,3 +326,39 @@ def test_local_search_window_rejects_large_S():
     with pytest.raises(pm.PMError) as ei:
         pm.local_search(E, method="window")
     assert ei.value.status == pm.PM_ERR_UNSUPPORTED
+
+
+# ------------------------------------------------------- fused Step 1 path --
+@pytest.mark.parametrize("N,M,C,rows", [(512, 16, 3, (100, 900)), (256, 16, 1, None), (192, 32, 1, (3, 30)),
+                                        (320, 16, 3, (0, 400))])
+def test_error_matrix_fused_loader_parity(N, M, C, rows):
+    # M*C % 16 == 0 and P % 64 == 0: the E kernel reads tiles straight from the images
+    I, T = pair("noise", N, M, C)
+    E = pm.error_matrix(dev(I), dev(T), M, rows=rows).cpu().numpy()
+    ref = oracle_E("noise", N, M, C)
+    assert (E == (ref if rows is None else ref[rows[0]:rows[1]])).all()
+
+
+def test_error_matrix_unaligned_images_fall_back_to_packing():
+    # image base pointers not 16-byte aligned -> packed path, same result
+    I, T = pair("smooth", 512, 16)
+    bufI = torch.empty(I.size + 16, dtype=torch.uint8, device=DEV)
+    bufT = torch.empty(T.size + 16, dtype=torch.uint8, device=DEV)
+    dI = bufI[1:1 + I.size].view(512, 512, 3)
+    dT = bufT[3:3 + T.size].view(512, 512, 3)
+    dI.copy_(dev(I))
+    dT.copy_(dev(T))
+    E = pm.error_matrix(dI, dT, 16).cpu().numpy()
+    assert (E == oracle_E("smooth", 512, 16)).all()
+
+
+def test_error_matrix_simulated_8_shards_config4():
+    # the row shards an 8-GPU job computes (dist.shard_rows) reassemble E exactly
+    from paper_conf_ipps_yangin17_b200 import dist as pdist
+    I, T = pair("smooth", 2048, 16)
+    dI, dT = dev(I), dev(T)
+    full = pm.error_matrix(dI, dT, 16)
+    for g in range(8):
+        b, e = pdist.shard_rows(16384, 8, g)
+        part = pm.error_matrix(dI, dT, 16, rows=(b, e))
+        assert torch.equal(part, full[b:e])
