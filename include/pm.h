@@ -50,8 +50,13 @@ typedef enum {
   PM_LS_CTA = 2,       /* one CTA runs every round on the device: r and the
                           maintained diagonal d in shared memory, E gathered
                           from L2/HBM (S <= pm_ls_cta_max_S())                */
-  PM_LS_WINDOW = 3     /* one CTA, plus a shared-memory window of each slot's
+  PM_LS_WINDOW = 3,    /* one CTA, plus a shared-memory window of each slot's
                           upcoming E entries streamed ahead of the classes    */
+  PM_LS_PAIRWIN = 4    /* per round: a grid-wide kernel tabulates every pair's
+                          two terms of line 5 at the round's start, one CTA
+                          streams the class rows and patches swapped slots;
+                          rounds looped on the device (CUDA-graph WHILE node);
+                          40 <= S <= 2048 on this build                       */
 } pm_ls_method_t;
 
 const char* pm_status_string(pm_status_t s);

@@ -304,6 +304,8 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
       return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     case PM_LS_WINDOW:
       return run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+    case PM_LS_PAIRWIN:
+      return run_pairwin(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     default:
       return PM_ERR_UNSUPPORTED;
   }

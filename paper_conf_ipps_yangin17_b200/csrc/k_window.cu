@@ -444,6 +444,17 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
 
 int32_t ls_window_max_S() { return 2048; }
 
+cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int64_t ldp, int32_t S, int32_t m,
+                                int32_t ext, cudaStream_t st) {
+  const int64_t total = (int64_t)S * (m + ext);
+  int64_t blocks = (total + 255) / 256;
+  if (blocks > 148 * 8) blocks = 148 * 8;
+  if (blocks < 1) blocks = 1;
+  k_permute_cols<<<(unsigned)blocks, 256, 0, st>>>(E, ldE, Ep, ldp, S, m, ext);
+  note_launch();
+  return cudaGetLastError();
+}
+
 template <int K, int PPT, int MAXT>
 static pm_status_t launch_window_k(const int32_t* E, int64_t ldE, const int32_t* Ep, int64_t ldp, int32_t S,
                                    int32_t* perm, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,

@@ -107,6 +107,13 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
                              int32_t* used_method);
 int32_t ls_class_launches_per_round(int32_t S);
 int32_t ls_window_max_S();
+int32_t ls_pairwin_min_S();
+int32_t ls_pairwin_max_S();
+// Ep[t][pos] = E[t][2 pos mod m], pos in [0, m + ext) (sigma-permuted rows, k_window.cu)
+cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int64_t ldp, int32_t S, int32_t m,
+                                int32_t ext, cudaStream_t st);
+pm_status_t run_pairwin(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                        LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                        LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm,

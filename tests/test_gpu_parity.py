@@ -131,7 +131,13 @@ def test_error_matrix_config5_row_chunks_sampled():
 
 
 # ------------------------------------------------------------------ Alg. 2 --
+def _supported(method, S):
+    return not (method == "pairwin" and not (40 <= S <= 2048)) and not (method == "window" and S > 2048)
+
+
 def _check_ls(E_np, method, perm0=None, max_rounds=0):
+    if not _supported(method, E_np.shape[0]):
+        pytest.skip(f"{method} does not take S = {E_np.shape[0]}")
     ref = oracle.local_search(E_np, r0=perm0, max_rounds=max_rounds)
     E = dev(E_np)
     perm = dev(np.arange(E_np.shape[0], dtype=np.int32) if perm0 is None else perm0.astype(np.int32))
@@ -144,13 +150,13 @@ def _check_ls(E_np, method, perm0=None, max_rounds=0):
     return ref
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "shuffle", "transposition", "identical"])
 def test_local_search_parity_config1(method, fam):
     _check_ls(oracle_E(fam, 128, 8), method)
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
 def test_local_search_parity_config2(method, fam):
     _check_ls(oracle_E(fam, 512, 16), method)
@@ -162,21 +168,21 @@ def test_local_search_parity_config3(method):
     assert ref[1] >= 3
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("N,M,C", [(90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (30, 10, 3), (64, 64, 1)])
 def test_local_search_parity_ragged_and_odd(method, N, M, C):
     # S = 81, 49, 9 are odd (the fixed point idles, reading R9); S = 1 trivial
     _check_ls(oracle_E("smooth", N, M, C), method)
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
 def test_local_search_resume_from_any_bijection(method):
     E = oracle_E("noise", 128, 8)
     rng = np.random.default_rng(3)
     _check_ls(E, method, perm0=rng.permutation(256).astype(np.int32))
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
 def test_local_search_max_rounds_then_resume(method):
     E_np = oracle_E("smooth", 512, 16)
     ref = _check_ls(E_np, method, max_rounds=2)
@@ -184,7 +190,7 @@ def test_local_search_max_rounds_then_resume(method):
     _check_ls(E_np, method, perm0=ref[0])
 
 
-@pytest.mark.parametrize("method", ["window", "cta", "class"])
+@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
 def test_local_search_rejects_non_permutation(method):
     E = dev(oracle_E("smooth", 128, 8))
     bad = torch.arange(256, dtype=torch.int32, device=DEV)
@@ -206,6 +212,8 @@ def test_local_search_random_small_matrices():
         E = rng.integers(0, 4, size=(S, S)).astype(np.int32)
         for method in ("window", "cta", "class"):
             _check_ls(E, method)
+        if S >= 40:
+            _check_ls(E, "pairwin")
 
 
 def _two_opt_gpu(E, perm):
@@ -262,7 +270,7 @@ def test_cost_int64():
 
 
 # -------------------------------------------------------------- pipeline ----
-@pytest.mark.parametrize("method", ["auto", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "pairwin", "window", "cta", "class"])
 def test_photomosaic_pipeline_config2(method):
     I, T = pair("smooth", 512, 16)
     E_np = oracle_E("smooth", 512, 16)
@@ -309,16 +317,25 @@ def test_launch_count_increments():
     assert pm.launch_count() - n0 >= 5   # 2 pack + E + iota + search + cost
 
 
-@pytest.mark.parametrize("N,M", [(1600, 40), (1152, 32), (1440, 32)])
-def test_local_search_window_sizes(N, M):
-    # S = 1600, 1296, 2025 (the K = 4 window tier, S in (1024, 2048]), grayscale noise
-    _check_ls(oracle_E("noise", N, M, 1), "window")
+@pytest.mark.parametrize("method", ["window", "pairwin"])
+@pytest.mark.parametrize("N,M", [(1600, 40), (1152, 32), (1440, 32), (224, 32), (280, 40)])
+def test_local_search_window_sizes(N, M, method):
+    # S = 1600, 1296, 2025 (the second window tier, S in (1024, 2048]), 49, 49 -- grayscale noise
+    _check_ls(oracle_E("noise", N, M, 1), method)
 
 
-@pytest.mark.parametrize("S_side", [31, 33, 45])
-def test_local_search_window_odd_mid(S_side):
-    # odd S around the window tiers (961, 1089, 2025)
-    _check_ls(oracle_E("smooth", S_side * 4, 4, 3), "window")
+@pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "transposition", "identical", "shuffle"])
+@pytest.mark.parametrize("N,M", [(512, 16), (160, 8), (328, 8)])
+def test_local_search_pairwin_families(fam, N, M):
+    # S = 1024, 400, 1681 (odd)
+    _check_ls(oracle_E(fam, N, M), "pairwin")
+
+
+@pytest.mark.parametrize("method", ["window", "pairwin"])
+@pytest.mark.parametrize("S_side", [7, 31, 33, 45])
+def test_local_search_window_odd_mid(S_side, method):
+    # odd S around the window tiers (49, 961, 1089, 2025)
+    _check_ls(oracle_E("smooth", S_side * 4, 4, 3), method)
 
 
 def test_local_search_window_rejects_large_S():
