@@ -221,7 +221,10 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
 int32_t pm_ls_cta_max_S(void) { return ls_cta_max_S(); }
 
 int32_t pm_ls_auto_method(int32_t S) {
-  return (S <= ls_window_max_S()) ? PM_LS_WINDOW : (S <= ls_cta_max_S()) ? PM_LS_CTA : PM_LS_CLASS;
+  // measured on B200: WINDOW fastest up to its shared-memory limit; beyond it
+  // the graph of per-class kernels beats one CTA (whose gather rate is bounded
+  // by one SM: 2.4 vs 2.6 us/class at S = 4096, 3.3 vs 11.7 at S = 16384)
+  return (S <= ls_window_max_S()) ? PM_LS_WINDOW : PM_LS_CLASS;
 }
 
 pm_status_t pm_cost_async(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int64_t* d_cost,

@@ -10,7 +10,7 @@ from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
 
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["1", "2", "3"])]
 methods = sys.argv[2].split(",") if len(sys.argv) > 2 else ["window", "cta"]
-reps = int(os.environ.get("REPS", "5"))
+reps = max(1, int(os.environ.get("REPS", "5")))
 for cfg in cfgs:
     c = synth.CONFIGS[cfg]
     I, T = synth.config_pair(cfg, "smooth", 0)
