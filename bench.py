@@ -271,13 +271,24 @@ def bench_ours(args, rank, world, local_rank):
     used = pm.ls_auto_method(S) if args.method == "auto" else args.method
     ls_kernel = {"window": "k_ls_window (+ k_permute_cols)", "cta": "k_ls_cta",
                  "class": "k_ls_class x (S-1) per round (CUDA graph)"}[used]
+    traffic = {}
+    try:
+        traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+    except (OSError, ValueError):
+        pass
+
+    def _traffic(name):
+        t = traffic.get(name)
+        return None if not t else t["dram_read_bytes"] + t["dram_write_bytes"]
+
     roof_ls = {"kernel": f"{ls_kernel}: Alg. 2, all rounds", "bound": "hbm", "achieved": ls_gbs,
-               "peak": hbm_peak, "unit": "GB/s", "frac": ls_gbs / hbm_peak, "traffic": None,
+               "peak": hbm_peak, "unit": "GB/s", "frac": ls_gbs / hbm_peak,
+               "traffic": _traffic("k_ls_" + used) if used in ("window", "cta") else None,
                "peak_source": hbm_src, "algorithmic_bytes": ls_bytes,
                "note": "latency-bound dependency chain of S-1 class steps per round; bytes = rounds*S(S-1)/2*8"}
     roof_e = {"kernel": "k_sad (Eq. 1; Step 1 fused into its loader at S <= 4096)", "bound": "alu",
               "achieved": e_tops, "peak": alu_peak,
-              "unit": "T byte-absdiff/s", "frac": e_tops / alu_peak, "traffic": None,
+              "unit": "T byte-absdiff/s", "frac": e_tops / alu_peak, "traffic": _traffic("k_sad"),
               "peak_source": f"derived: 148 SM x {ALU_VABSDIFF4_PER_CLK_PER_SM} VABSDIFF4/clk x 4 B x {sm_max} MHz",
               "gpairs_per_s": S * S / (mean_e * 1e-3) / 1e9}
     dominant = roof_ls if mean_ls >= mean_e else roof_e
