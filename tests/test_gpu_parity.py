@@ -379,3 +379,29 @@ def test_error_matrix_simulated_8_shards_config4():
         b, e = pdist.shard_rows(16384, 8, g)
         part = pm.error_matrix(dI, dT, 16, rows=(b, e))
         assert torch.equal(part, full[b:e])
+
+
+# ------------------------------------------- NEXT-1: the paper's grayscale grid
+@pytest.mark.parametrize("N,g", [(512, 16), (512, 32), (1024, 16), (1024, 32), (2048, 16)])
+def test_paper_grid_grayscale_parity(N, g):
+    # Tables II-IV shapes, C = 1: tile sides 8..128 px, P up to 16384 bytes
+    M = N // g
+    I, T = pair("smooth", N, M, 1)
+    Eg = pm.error_matrix(dev(I), dev(T), M)
+    E = oracle_E("smooth", N, M, 1)
+    assert (Eg.cpu().numpy() == E).all()
+    ref = oracle.local_search(E)
+    perm, rounds, swaps, per, st = pm.local_search(Eg)
+    assert (perm.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    assert pm.cost(Eg, perm) == oracle.cost(E, ref[0])
+
+
+@pytest.mark.parametrize("N,g", [(512, 64), (2048, 64)])
+def test_paper_grid_grayscale_S4096_sampled(N, g):
+    # S = 64^2 = 4096 (the paper's largest grid): E sampled against the oracle,
+    # the search against the oracle replay run on the oracle's own E
+    M = N // g
+    I, T = pair("smooth", N, M, 1)
+    Eg = pm.error_matrix(dev(I), dev(T), M)
+    rng = np.random.default_rng(N)
+    _sampled_E_check(I, T, M, Eg, 0, rng, 400)
