@@ -197,6 +197,14 @@ pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
                                 int32_t* h_perm, int32_t* h_rounds, int64_t* h_swaps,
                                 int64_t* h_cost, pm_stream_t stream);
 
+/* The resulting photomosaic R (Sec. V P:247 "writes the resulting
+ * photomosaic image to the global memory"): target slot u of d_out shows
+ * input tile r[u] = d_perm[u] of d_input, pixel for pixel (raster tiles,
+ * (y, x, c) order, reading R4).  d_input / d_out: u8 [N][N][C] HWC, distinct
+ * buffers; d_perm: int32 [S] (not validated as a bijection here).  Async. */
+pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, const int32_t* d_perm,
+                      uint8_t* d_out, pm_stream_t stream);
+
 /* Number of this library's kernel launches enqueued by the calling process
  * so far (for launch accounting in benchmarks). */
 int64_t pm_launch_count(void);

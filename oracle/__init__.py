@@ -21,6 +21,7 @@ local_search_np(E, r0=None)         Algorithm 2, vectorised per group (second fo
 serial_local_search(E)              Algorithm 1, P:118-129        (C)
 cost(E, r)                          Eq. (2), P:63                 (C)
 hungarian(E)                        Sec. III, Kuhn-Munkres P:102  (C, with dual certificate)
+render(I, M, r)                     the photomosaic image R, P:61/P:247 (C)
 brute_force(E)                      Eq. (3), all S! rearrangements (Python, S <= 8)
 
 Pins (tests/test_oracle_*.py) tie each of these to something other than
@@ -83,6 +84,8 @@ def _load():
     lib.or_serial_local_search.restype = ctypes.c_int32
     lib.or_hungarian.argtypes = [_I32P, ctypes.c_int64, ctypes.c_int32, _I32P, _I64P, _I64P, _I64P]
     lib.or_hungarian.restype = ctypes.c_int32
+    lib.or_render.argtypes = [_U8P, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _I32P, _U8P]
+    lib.or_render.restype = None
     lib.or_num_threads.argtypes = []
     lib.or_num_threads.restype = ctypes.c_int32
     lib.or_set_num_threads.argtypes = [ctypes.c_int32]
@@ -240,6 +243,16 @@ def serial_local_search(E: np.ndarray, r0: np.ndarray | None = None, max_rounds:
     st = _load().or_serial_local_search(_p(E, _I32P), E.shape[1], S, _p(r, _I32P), int(max_rounds),
                                         ctypes.byref(rounds), ctypes.byref(swaps))
     return r, int(rounds.value), int(swaps.value), int(st)
+
+
+# ---------------------------------------------------------------- render ---
+def render(I: np.ndarray, M: int, r: np.ndarray) -> np.ndarray:
+    """The photomosaic R: slot u shows input tile r[u]."""
+    a, N, C = _img(I)
+    r = np.ascontiguousarray(r, dtype=np.int32)
+    out = np.empty_like(a)
+    _load().or_render(_p(a, _U8P), N, M, C, _p(r, _I32P), _p(out, _U8P))
+    return out if np.asarray(I).ndim == 3 else out[:, :, 0]
 
 
 # ---------------------------------------------------------------- Sec. III -

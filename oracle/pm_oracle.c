@@ -279,6 +279,23 @@ int32_t or_hungarian(const int32_t* E, int64_t ldE, int32_t S, int32_t* r, int64
   return 0;
 }
 
+/* ------------------------------------------------------------------------ */
+/* The resulting photomosaic R ("writes the resulting photomosaic
+ * image"): target slot u of R shows input tile r[u], pixel by pixel, in the
+ * same raster tile geometry as Step 1 (reading R4).                         */
+void or_render(const uint8_t* I, int32_t N, int32_t M, int32_t C, const int32_t* r, uint8_t* R) {
+  int64_t g = N / M, S = g * g;
+  for (int64_t u = 0; u < S; ++u) {
+    int64_t t = r[u];
+    int64_t uy = u / g, ux = u % g, ty = t / g, tx = t % g;
+    for (int64_t y = 0; y < M; ++y)
+      for (int64_t x = 0; x < M; ++x)
+        for (int64_t c = 0; c < C; ++c)
+          R[((uy * M + y) * (int64_t)N + ux * M + x) * C + c] =
+              I[((ty * M + y) * (int64_t)N + tx * M + x) * C + c];
+  }
+}
+
 int32_t or_num_threads(void) {
 #ifdef _OPENMP
   return omp_get_max_threads();

@@ -63,6 +63,38 @@ cudaError_t launch_pack(const uint8_t* img, int32_t N, int32_t M, int32_t C, uin
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------------- render R ---
+// The photomosaic: target slot u of R shows input tile r[u].
+// One thread per output byte (coalesced writes; the reads are row segments of
+// the source tile).
+__global__ void k_render(const uint8_t* __restrict__ img, int32_t N, int32_t M, int32_t C,
+                         const int32_t* __restrict__ perm, uint8_t* __restrict__ out) {
+  const int32_t g = N / M;
+  const int64_t total = (int64_t)N * N * C;
+  const int64_t rowb = (int64_t)N * C;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t py = i / rowb;
+    const int32_t rem = (int32_t)(i - py * rowb);
+    const int32_t px = rem / C, c = rem - px * C;
+    const int32_t uy = (int32_t)(py / M), y = (int32_t)(py - (int64_t)uy * M);
+    const int32_t ux = px / M, x = px - ux * M;
+    const int32_t t = __ldg(perm + (int64_t)uy * g + ux);
+    const int32_t ty = t / g, tx = t - ty * g;
+    out[i] = __ldg(img + ((int64_t)(ty * M + y) * N + tx * M + x) * C + c);
+  }
+}
+
+cudaError_t launch_render(const uint8_t* img, int32_t N, int32_t M, int32_t C, const int32_t* perm,
+                          uint8_t* out, cudaStream_t st) {
+  const int64_t total = (int64_t)N * N * C;
+  int64_t blocks = (total + 255) / 256;
+  if (blocks > 148 * 16) blocks = 148 * 16;
+  if (blocks < 1) blocks = 1;
+  k_render<<<(unsigned)blocks, 256, 0, st>>>(img, N, M, C, perm, out);
+  note_launch();
+  return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- Step 2 ---
 namespace sad {
 constexpr int kThreads = 256;

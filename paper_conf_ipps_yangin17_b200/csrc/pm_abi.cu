@@ -318,6 +318,14 @@ pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
   return PM_OK;
 }
 
+pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, const int32_t* d_perm,
+                      uint8_t* d_out, pm_stream_t stream) {
+  if (!valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  if (!d_input || !d_perm || !d_out || d_out == d_input) return PM_ERR_INVALID;
+  PM_CUDA_TRY(launch_render(d_input, N, M, C, d_perm, d_out, (cudaStream_t)stream));
+  return PM_OK;
+}
+
 int64_t pm_launch_count(void) { return g_launches.load(); }
 
 }  // extern "C"

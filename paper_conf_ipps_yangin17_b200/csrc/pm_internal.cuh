@@ -84,6 +84,8 @@ cudaError_t launch_pack(const uint8_t* img, int32_t N, int32_t M, int32_t C, uin
                         int64_t ld_tiles, int32_t tile_begin, int32_t tile_end, cudaStream_t st);
 cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
                        int32_t P, int32_t* E, int64_t ldE, cudaStream_t st);
+cudaError_t launch_render(const uint8_t* img, int32_t N, int32_t M, int32_t C, const int32_t* perm,
+                          uint8_t* out, cudaStream_t st);
 // Step 1 fused into the E kernel's loader (no packed tiles): requires
 // sad_image_ok (a tile row is a whole number of 16-byte pieces, P % 64 == 0).
 bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C);

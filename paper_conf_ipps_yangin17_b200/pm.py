@@ -46,6 +46,7 @@ _SIGS = [
     ("pm_photomosaic", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _P, _I64, _P, _I32, _P, _P, _P, _P]),
     ("pm_photomosaic_async", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _P, _I64, _P, _I32, _P, _P]),
     ("pm_photomosaic_host", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _I32, _P, _P, _P, _P, _P]),
+    ("pm_render", ctypes.c_int, [_P, _I32, _I32, _I32, _P, _P, _P]),
     ("pm_launch_count", _I64, []),
 ]
 
@@ -282,6 +283,17 @@ def photomosaic_host(I: np.ndarray, T: np.ndarray, M: int, method: str = "auto",
                                      ctypes.byref(rounds), ctypes.byref(swaps), ctypes.byref(c), _stream(stream)),
            "pm_photomosaic_host")
     return perm_out, int(rounds.value), int(swaps.value), int(c.value)
+
+
+def render(I, M: int, perm, out=None, stream=None):
+    """pm_render: the photomosaic image R, slot u showing input tile perm[u]."""
+    torch = _torch()
+    img = _dev_u8_image(I)
+    N, C = img.shape[0], img.shape[2]
+    if out is None:
+        out = torch.empty_like(img)
+    _check(lib().pm_render(img.data_ptr(), N, M, C, perm.data_ptr(), out.data_ptr(), _stream(stream)), "pm_render")
+    return out if I.dim() == 3 else out[:, :, 0]
 
 
 def launch_count() -> int:

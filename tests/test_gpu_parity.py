@@ -405,3 +405,20 @@ def test_paper_grid_grayscale_S4096_sampled(N, g):
     Eg = pm.error_matrix(dev(I), dev(T), M)
     rng = np.random.default_rng(N)
     _sampled_E_check(I, T, M, Eg, 0, rng, 400)
+
+
+# ------------------------------------------------- NEXT-3: render R --
+@pytest.mark.parametrize("N,M,C", [(128, 8, 3), (90, 10, 3), (200, 5, 1)])
+def test_render_parity(N, M, C):
+    I, T = pair("noise", N, M, C)
+    S = (N // M) ** 2
+    perm = np.random.default_rng(S).permutation(S).astype(np.int32)
+    R = pm.render(dev(I), M, dev(perm)).cpu().numpy()
+    assert R.shape == I.shape and (R == oracle.render(I, M, perm)).all()
+
+
+def test_render_transposition_reproduces_target():
+    # closed form: Alg. 2 solves a transposition exactly, so R == T bit for bit
+    I, T = pair("transposition", 512, 16)
+    perm, rounds, swaps, cost, E = pm.photomosaic(dev(I), dev(T), 16)
+    assert cost == 0 and (pm.render(dev(I), 16, perm).cpu().numpy() == T).all()

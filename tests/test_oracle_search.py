@@ -188,3 +188,28 @@ def test_alg1_hand_trace():
     E = np.array([[3, 7, 2, 8], [6, 1, 5, 4], [2, 9, 6, 3], [7, 4, 1, 5]], dtype=np.int32)
     r, k, s, st = oracle.serial_local_search(E)
     assert r.tolist() == [2, 1, 0, 3] and (k, s) == (2, 1)
+
+
+def test_render_identity_and_hand_example():
+    # slot u of R shows input tile r[u]
+    img = np.arange(16, dtype=np.uint8).reshape(4, 4)          # tiles [0,1,4,5] [2,3,6,7] [8,9,12,13] [10,11,14,15]
+    assert (oracle.render(img, 2, np.arange(4)) == img).all()
+    R = oracle.render(img, 2, np.array([3, 2, 1, 0]))
+    assert R.tolist() == [[10, 11, 8, 9], [14, 15, 12, 13], [2, 3, 0, 1], [6, 7, 4, 5]]
+
+
+def test_render_optimum_of_shuffle_reproduces_target():
+    # T is a tile permutation of I, so the optimum (cost 0) renders T exactly
+    I, T = synth.make_pair("shuffle", 96, 8, 3, seed=4)
+    E = oracle.error_matrix(I, T, 8)
+    r, c, p, q = oracle.hungarian(E)
+    assert c == 0 and (oracle.render(I, 8, r) == T).all()
+
+
+def test_render_cost_identity():
+    # Eq. (2): the total error equals the pixelwise L1 distance of R and T
+    I, T = synth.make_pair("smooth", 64, 8, 3, seed=5)
+    E = oracle.error_matrix(I, T, 8)
+    r = oracle.local_search(E)[0]
+    R = oracle.render(I, 8, r)
+    assert oracle.cost(E, r) == int(np.abs(R.astype(np.int64) - T.astype(np.int64)).sum())
