@@ -169,6 +169,7 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
   }
   for (int32_t i = tid; i < S * K; i += T) s_SW[i] = p->SWg[i];
   if (tid < 4) s_ctl[tid] = INT32_MAX;
+  if (tid == 4 || tid == 5) s_ctl[tid] = 0;    // [4]: swapped since last compaction, [5]: dirty-list size
 
   auto wrap = [&](int32_t q) -> int32_t { if (q < 0) q += m; if (q >= m) q -= m; return q; };
   // (array, column) of regular slot x at class c; returns -1 if it idles (odd S)
@@ -215,8 +216,10 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
 #endif
     // ---- slots swapped earlier this round: re-derive their entries (and SW
     // for those swapped in the previous window) from their current rows
-    // compact the round-dirty regular slots into s_dl (warp ballots + prefix)
-    {
+    // compact the round-dirty regular slots into s_dl (warp ballots + prefix),
+    // only if some slot swapped since the last compaction (block-uniform flag)
+    int32_t tot = s_ctl[5];
+    if (s_ctl[4]) {
       const int nw = T >> 5, wid_ = tid >> 5;
       const int32_t chunk = (nreg + nw - 1) / nw;
       const int32_t x0 = wid_ * chunk, x1 = min(nreg, x0 + chunk);
@@ -228,7 +231,8 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
       int* red = s_ctl + 8;
       if (lane == 0) red[wid_] = cnt;
       __syncthreads();
-      int32_t off = 0, tot = 0;
+      int32_t off = 0;
+      tot = 0;
       for (int i = 0; i < nw; ++i) { const int32_t ci = red[i]; off += i < wid_ ? ci : 0; tot += ci; }
       for (int32_t xb = x0; xb < x1; xb += 32) {
         const int32_t x = xb + lane;
@@ -238,6 +242,9 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
         off += __popc(bm);
       }
       __syncthreads();
+      if (tid == 0) { s_ctl[4] = 0; s_ctl[5] = tot; }
+    }
+    {
       // ---- re-derive their entries (and SW for those swapped in the previous window)
       constexpr int U = 8;                     // loads in flight per thread
       const int32_t items = tot * K;
@@ -371,6 +378,7 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
         }
       }
       const int any = __syncthreads_or(fired);
+      if (any && tid == 0) s_ctl[4] = 1;
       if (cend - c <= 1 && !any) B = 2;
       c = cc + 1;
     }
