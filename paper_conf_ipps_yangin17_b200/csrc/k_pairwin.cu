@@ -131,7 +131,10 @@ struct PwSmem {
 // One round of Algorithm 2 in one CTA (lines 2-10).
 template <int K>
 __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) {
-  if (p->out->status != PM_OK) return;
+  __shared__ int s_status;                      // block-uniform early exit (no divergent barrier)
+  if (threadIdx.x == 0) s_status = (int)p->out->status;
+  __syncthreads();
+  if (s_status != PM_OK) return;
   extern __shared__ __align__(16) int32_t sm[];
   const int32_t S = p->S, npr = p->npr;
   const Classes cl(S);

@@ -1,0 +1,24 @@
+"""Small workload for compute-sanitizer: every kernel of libpm once (configs 1
+and a ragged odd shape), results checked against the oracle."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import oracle
+from paper_conf_ipps_yangin17_b200 import pm, synth
+for (N, M, C) in [(128, 8, 3), (90, 10, 3)]:
+    I, T = synth.make_pair("smooth", N, M, C, seed=1)
+    dI, dT = torch.from_numpy(I).cuda(), torch.from_numpy(T).cuda()
+    E = pm.error_matrix(dI, dT, M)
+    Er = oracle.error_matrix(I, T, M)
+    assert (E.cpu().numpy() == Er).all()
+    ref = oracle.local_search(Er)
+    methods = os.environ.get("METHODS", "window,cta,class,pairwin").split(",")
+    for meth in methods:
+        if meth == "pairwin" and E.shape[0] < 40:
+            continue
+        perm, rounds, swaps, per, st = pm.local_search(E, method=meth)
+        assert (perm.cpu().numpy() == ref[0]).all() and rounds == ref[1], meth
+    c = pm.cost(E, perm)
+    R = pm.render(dI, M, perm)
+    t = pm.pack_tiles(dI, M)
+print("sanitize workload ok")
