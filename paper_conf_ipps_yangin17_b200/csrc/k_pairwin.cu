@@ -124,13 +124,13 @@ __device__ __forceinline__ void pw_cp16(int32_t* smem, const int32_t* gmem) {
 template <int K>
 struct PwSmem {
   static size_t bytes(int32_t S, int32_t npr) {
-    return sizeof(int32_t) * (((size_t)S * 6 + (size_t)S * K + 3) / 4 * 4 + (size_t)4 * K * npr + 64);
+    return sizeof(int32_t) * (((((size_t)S * 6 + 3) / 4 * 4) + (size_t)S * K + 3) / 4 * 4 + (size_t)4 * K * npr + 64);
   }
 };
 
 // One round of Algorithm 2 in one CTA (lines 2-10).
-template <int K>
-__global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) {
+template <int K, int MAXT>
+__global__ void __launch_bounds__(MAXT, 1) k_pw_round(PwParams* __restrict__ p) {
   __shared__ int s_status;                      // block-uniform early exit (no divergent barrier)
   if (threadIdx.x == 0) s_status = (int)p->out->status;
   __syncthreads();
@@ -153,8 +153,8 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
   int32_t* s_sig = s_last + S;           // sigma(x)
   int32_t* s_gen = s_sig + S;            // window id of x's last swap this round (-1: none)
   int32_t* s_dl = s_gen + S;             // this window's list of slots swapped earlier this round
-  int32_t* s_SW = s_dl + S;              // [S][K]
-  int32_t* s_T = sm + ((size_t)S * 6 + (size_t)S * K + 3) / 4 * 4;   // [2 buf][2 (U,V)][K][npr], 16-B aligned
+  int32_t* s_SW = sm + ((size_t)S * 6 + 3) / 4 * 4;                  // [S][K], 16-B aligned
+  int32_t* s_T = sm + ((((size_t)S * 6 + 3) / 4 * 4) + (size_t)S * K + 3) / 4 * 4;   // [2 buf][2 (U,V)][K][npr], 16-B aligned
   int32_t* s_ctl = s_T + (size_t)4 * K * npr;
   const int32_t tsz = K * npr;           // one array of one buffer
 
@@ -170,7 +170,12 @@ __global__ void __launch_bounds__(1024, 1) k_pw_round(PwParams* __restrict__ p) 
     s_sig[x] = x < m ? pw_sigma(x, m, H) : 0;
     s_gen[x] = -1;
   }
-  for (int32_t i = tid; i < S * K; i += T) s_SW[i] = p->SWg[i];
+  {                                            // SW: 16-byte cp.async (S*K ints, 16-B aligned)
+    const int32_t n16 = S * K / 4;
+    for (int32_t i = tid; i < n16; i += T) pw_cp16(s_SW + 4 * i, p->SWg + 4 * i);
+    for (int32_t i = n16 * 4 + tid; i < S * K; i += T) s_SW[i] = p->SWg[i];
+    asm volatile("cp.async.commit_group;\n" ::);
+  }
   if (tid < 4) s_ctl[tid] = INT32_MAX;
   if (tid == 4 || tid == 5) s_ctl[tid] = 0;    // [4]: swapped since last compaction, [5]: dirty-list size
 
@@ -441,7 +446,8 @@ static cudaError_t pw_build_graph(int32_t S, int32_t npr, PwGraph& out) {
   cudaError_t e = cudaMalloc(&out.dparams, sizeof(PwParams));
   if (e != cudaSuccess) return e;
   const size_t smem = PwSmem<K>::bytes(S, npr);
-  if ((e = cudaFuncSetAttribute(k_pw_round<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
+  constexpr int MAXT = K == 16 ? 512 : 1024;       // S <= 1024 runs 512 threads: 128 registers, no spills
+  if ((e = cudaFuncSetAttribute(k_pw_round<K, MAXT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
     return e;
   cudaGraph_t g = nullptr;
   if ((e = cudaGraphCreate(&g, 0)) != cudaSuccess) return e;
@@ -465,7 +471,7 @@ static cudaError_t pw_build_graph(int32_t S, int32_t npr, PwGraph& out) {
   if (blocks > 148 * 8) blocks = 148 * 8;
   if (blocks < 1) blocks = 1;
   k_pw_tables<<<blocks, 256, 0, cs>>>(out.dparams);
-  k_pw_round<K><<<1, pw_threads<K>(S), smem, cs>>>(out.dparams);
+  k_pw_round<K, MAXT><<<1, pw_threads<K>(S), smem, cs>>>(out.dparams);
   k_pw_round_end<<<1, 1, 0, cs>>>(out.dparams, h);
   cudaGraph_t captured = body;
   e = cudaStreamEndCapture(cs, &captured);
