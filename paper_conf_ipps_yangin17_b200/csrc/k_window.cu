@@ -230,6 +230,7 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
   int status = PM_OK;
   uint32_t batch = 0;
   int32_t wid = -1;
+  bool dense = true;        // round 0, and rounds after one with > ncls/2 swaps (measured: B = 1 wins there)
 #ifdef PM_LS_PROFILE
   long long t_round = clock64();
   int32_t n_apply = 0, n_spec = 0;
@@ -259,6 +260,7 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
       int32_t* first_slot = s_ctl + (batch % 3);
       if (tid == 0) s_ctl[(batch + 1) % 3] = INT32_MAX;
       ++batch;
+      if (dense) B = 1;                                // dense round: speculation only wastes work
       const int32_t cend = min(c + B, wb + jmax);
       int32_t cc = c;
 #ifdef PM_LS_PROFILE
@@ -436,6 +438,7 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     if (rs == 0) break;
     if (max_rounds > 0 && rounds >= max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
     B = 1;
+    dense = rs > cl.ncls / 2;
   }
   __syncthreads();
   for (int32_t u = tid; u < S; u += T) perm[u] = s_r[u];

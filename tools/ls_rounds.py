@@ -4,7 +4,7 @@ import ctypes, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 from paper_conf_ipps_yangin17_b200 import pm, synth
-pm.LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libpm_prof.so")
+pm.LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), os.environ.get("PMLIB", "libpm_prof.so"))
 cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 method = sys.argv[2] if len(sys.argv) > 2 else "window"
 c = synth.CONFIGS[cfg]
