@@ -205,6 +205,30 @@ pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
 pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, const int32_t* d_perm,
                       uint8_t* d_out, pm_stream_t stream);
 
+/* The paper's optimization algorithm (Sec. III): the best
+ * rearrangement R* (Eq. 3), i.e. a minimum-weight perfect matching of
+ * the complete bipartite graph input tiles x target slots with
+ * w_{u,v} = E[u][v], which the paper computes on the CPU with Blossom V
+ * (P:102).  Here an exact GPU eps-scaling auction on the integer weights
+ * scaled by S + 1, finishing at eps = 1 (reading R16).
+ *   d_E     : int32 [S][ld_E] (rows = input tiles), entries in [0, 2^24)
+ *             (checked on the device: PM_ERR_INVALID after the launch if not).
+ *   d_perm  : int32 [S], out: r[v] = input tile at target slot v, with
+ *             sum_v E[r[v]][v] minimal over all bijections.  When several
+ *             bijections are optimal, which one is returned is unspecified
+ *             (deterministic for a given device and input).
+ *   d_price : int64 [S] or NULL, out: the final object prices p[v], a
+ *             certificate: with C = (S + 1) * E, every u = r[v] satisfies
+ *             C[u][v] + p[v] <= min_w (C[u][w] + p[w]) + 1.
+ *   h_rounds: bidding rounds executed (nullable).
+ *   h_cost  : sum_v E[r[v]][v] (int64, nullable).
+ * S <= 65536; needs cooperative launch (PM_ERR_UNSUPPORTED otherwise).
+ * PM_ERR_NOT_CONVERGED if the internal round cap (2^22) is hit.
+ * Synchronises `stream`. */
+pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                  int64_t* d_price, int32_t* h_rounds, int64_t* h_cost,
+                                  pm_stream_t stream);
+
 /* Number of this library's kernel launches enqueued by the calling process
  * so far (for launch accounting in benchmarks). */
 int64_t pm_launch_count(void);

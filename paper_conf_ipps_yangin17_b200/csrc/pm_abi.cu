@@ -326,6 +326,24 @@ pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, c
   return PM_OK;
 }
 
+pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm, int64_t* d_price,
+                                  int32_t* h_rounds, int64_t* h_cost, pm_stream_t stream) {
+  if (!d_E || !d_perm || S < 1 || ld_E < S) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  DevBuf buf;
+  buf.st = st;
+  if (h_cost) PM_CUDA_TRY(pm::scratch_alloc(&buf.p, sizeof(int64_t), st));
+  int32_t stats[2] = {0, 0};
+  const pm_status_t s = run_assignment(d_E, ld_E, S, d_perm, d_price, reinterpret_cast<int64_t*>(buf.p), stats, st);
+  if (h_rounds) *h_rounds = stats[0];
+  if (s != PM_OK) return s;
+  if (h_cost) {
+    PM_CUDA_TRY(cudaMemcpyAsync(h_cost, buf.p, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+    PM_CUDA_TRY(cudaStreamSynchronize(st));
+  }
+  return PM_OK;
+}
+
 int64_t pm_launch_count(void) { return g_launches.load(); }
 
 }  // extern "C"

@@ -120,5 +120,9 @@ pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, 
                        LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm,
                         int64_t* d_cost, cudaStream_t st);
+// Exact min-weight perfect matching by eps-scaling auction (k_assign.cu).
+// h_stats (nullable): {bidding rounds, phases}.  Synchronises st.
+pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* perm, int64_t* price_out,
+                           int64_t* cost_out_dev, int32_t* h_stats, cudaStream_t st);
 
 }  // namespace pm

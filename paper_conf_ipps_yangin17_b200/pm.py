@@ -47,6 +47,7 @@ _SIGS = [
     ("pm_photomosaic_async", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _P, _I64, _P, _I32, _P, _P]),
     ("pm_photomosaic_host", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _I32, _P, _P, _P, _P, _P]),
     ("pm_render", ctypes.c_int, [_P, _I32, _I32, _I32, _P, _P, _P]),
+    ("pm_optimal_assignment", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P, _P, _P]),
     ("pm_launch_count", _I64, []),
 ]
 
@@ -294,6 +295,25 @@ def render(I, M: int, perm, out=None, stream=None):
         out = torch.empty_like(img)
     _check(lib().pm_render(img.data_ptr(), N, M, C, perm.data_ptr(), out.data_ptr(), _stream(stream)), "pm_render")
     return out if I.dim() == 3 else out[:, :, 0]
+
+
+# ------------------------------------------------- optimum (Sec. III) ------
+def optimal_assignment(E, perm=None, price=None, stream=None):
+    """pm_optimal_assignment: the best rearrangement R* (Eq. 3) by an exact GPU
+    auction.  Returns (perm, cost, rounds, price); price (int64 CUDA [S]) is the
+    eps-CS certificate for the costs (S + 1) * E."""
+    torch = _torch()
+    _dev(E, torch.int32)
+    S = E.shape[0]
+    if perm is None:
+        perm = torch.empty(S, dtype=torch.int32, device=E.device)
+    if price is None:
+        price = torch.empty(S, dtype=torch.int64, device=E.device)
+    rounds, c = ctypes.c_int32(0), ctypes.c_int64(0)
+    _check(lib().pm_optimal_assignment(E.data_ptr(), E.stride(0), S, perm.data_ptr(), price.data_ptr(),
+                                       ctypes.byref(rounds), ctypes.byref(c), _stream(stream)),
+           "pm_optimal_assignment")
+    return perm, int(c.value), int(rounds.value), price
 
 
 def launch_count() -> int:
