@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--family", default="smooth")
-    ap.add_argument("--method", default="auto", choices=["auto", "class", "cta", "window"])
+    ap.add_argument("--method", default="auto", choices=["auto", "class", "cta", "window", "pairwin"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="budget of the cpu_baseline sample")
     ap.add_argument("--e2e-steps", type=int, default=10)

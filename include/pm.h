@@ -216,7 +216,8 @@ pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, c
  *   d_perm  : int32 [S], out: r[v] = input tile at target slot v, with
  *             sum_v E[r[v]][v] minimal over all bijections.  When several
  *             bijections are optimal, which one is returned is unspecified
- *             (deterministic for a given device and input).
+ *             and may differ between calls (the bidder lists are built with
+ *             atomics); the cost never does.
  *   d_price : int64 [S] or NULL, out: the final object prices p[v], a
  *             certificate: with C = (S + 1) * E, every u = r[v] satisfies
  *             C[u][v] + p[v] <= min_w (C[u][w] + p[w]) + 1.
