@@ -230,8 +230,11 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
                                   int64_t* d_price, int32_t* h_rounds, int64_t* h_cost,
                                   pm_stream_t stream);
 
-/* Number of this library's kernel launches enqueued by the calling process
- * so far (for launch accounting in benchmarks). */
+/* Number of this library's kernel launches by the calling process so far
+ * (for launch accounting in benchmarks): host-side launches plus the kernels
+ * that device-side graph loops (CLASS / PAIRWIN rounds, sparse rounds)
+ * launched, which count themselves on the device -- so this call reads a
+ * device counter back and synchronises with the devices it has used. */
 int64_t pm_launch_count(void);
 
 #ifdef __cplusplus

@@ -49,6 +49,7 @@ struct PwParams {
   unsigned long long round_swaps;
   LsResult* out;
   int64_t* per_round;
+  unsigned long long* launches;   // device-side launch counter (graph kernels)
 };
 
 __global__ void k_pw_set_params(PwParams* dst, PwParams src) { *dst = src; }
@@ -74,6 +75,7 @@ __device__ __forceinline__ int32_t pw_sigma(int32_t x, int32_t m, int32_t H) {
 
 // Round-start tables (grid-wide).
 __global__ void __launch_bounds__(256) k_pw_tables(const PwParams* __restrict__ p) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p->launches, 1ull);
   if (p->out->status != PM_OK) return;
   const Classes cl(p->S);
   const int32_t S = p->S, npr = p->npr, K = p->K, m = cl.m, H = cl.half;
@@ -100,6 +102,7 @@ __global__ void __launch_bounds__(256) k_pw_tables(const PwParams* __restrict__ 
 
 // Alg. 2 line 11 (+ the max_rounds cap): decide whether the while-node loops.
 __global__ void k_pw_round_end(PwParams* p, cudaGraphConditionalHandle h) {
+  atomicAdd(p->launches, 1ull);
   LsResult* o = p->out;
   unsigned cont = 0;
   if (o->status == PM_OK) {
@@ -131,6 +134,7 @@ struct PwSmem {
 // One round of Algorithm 2 in one CTA (lines 2-10).
 template <int K, int MAXT>
 __global__ void __launch_bounds__(MAXT, 1) k_pw_round(PwParams* __restrict__ p) {
+  if (threadIdx.x == 0) atomicAdd(p->launches, 1ull);
   __shared__ int s_status;                      // block-uniform early exit (no divergent barrier)
   if (threadIdx.x == 0) s_status = (int)p->out->status;
   __syncthreads();
@@ -524,6 +528,8 @@ pm_status_t run_pairwin(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm,
   hp.TU = TU; hp.TV = TV; hp.SWg = SWg; hp.S = S; hp.npr = npr; hp.K = K;
   hp.max_rounds = max_rounds; hp.max_log = max_log; hp.round_swaps = 0;
   hp.out = dev_out; hp.per_round = dev_per_round;
+  hp.launches = device_launch_counter();
+  if (!hp.launches) return PM_ERR_CUDA;
   k_pw_set_params<<<1, 1, 0, st>>>(pg.dparams, hp);
   const int blocks = (S + 255) / 256;
   k_pw_check_init<<<blocks, 256, 0, st>>>(pg.dparams);

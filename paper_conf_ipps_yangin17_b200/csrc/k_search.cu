@@ -35,10 +35,12 @@ struct LsParams {
   int32_t S;
   int32_t max_rounds;
   int32_t max_log;
-  int32_t pad;
+  int32_t sparse_T;    // hand over to sparse rounds after a round with <= sparse_T swaps
   unsigned long long round_swaps;
   LsResult* out;
   int64_t* per_round;
+  int32_t* handoff;    // SpParams::pending, or NULL
+  unsigned long long* launches;   // device-side launch counter (graph kernels)
 };
 
 // ------------------------------------------------------------- CLASS -----
@@ -66,6 +68,7 @@ __global__ void k_ls_check_seen(LsParams* p) {
 
 // One colour class P_{c+1}: every pair concurrently (Alg. 2 line 4).
 __global__ void __launch_bounds__(256) k_ls_class(const LsParams* __restrict__ p, int32_t c) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p->launches, 1ull);
   if (p->out->status != PM_OK) return;
   const Classes cl(p->S);
   const int32_t k = blockIdx.x * blockDim.x + threadIdx.x;
@@ -91,6 +94,7 @@ __global__ void __launch_bounds__(256) k_ls_class(const LsParams* __restrict__ p
 __global__ void k_ls_round_end(LsParams* p, cudaGraphConditionalHandle h) {
   LsResult* o = p->out;
   unsigned cont = 0;
+  atomicAdd(p->launches, 1ull);
   if (o->status == PM_OK) {
     const int64_t sw = (int64_t)p->round_swaps;
     p->round_swaps = 0;
@@ -99,6 +103,7 @@ __global__ void k_ls_round_end(LsParams* p, cudaGraphConditionalHandle h) {
     o->swaps += sw;
     if (sw > 0) {
       if (p->max_rounds > 0 && o->rounds >= p->max_rounds) o->status = PM_ERR_NOT_CONVERGED;
+      else if (p->handoff && sw <= p->sparse_T) *p->handoff = 1;   // quiet: sparse rounds take over
       else cont = 1;
     }
   }
@@ -149,7 +154,8 @@ static cudaError_t build_class_graph(int32_t S, cudaStream_t st, ClassGraph& out
 }
 
 static pm_status_t run_class(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
-                             LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
+                             LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                             int32_t* handoff, int32_t sparse_T) {
   int dev = 0;
   PM_CUDA_TRY(cudaGetDevice(&dev));
   ClassGraph cg;
@@ -171,15 +177,16 @@ static pm_status_t run_class(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   hp.E = E; hp.ldE = ldE; hp.r = perm; hp.d = scratch; hp.seen = scratch + S;
   hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
   hp.round_swaps = 0; hp.out = dev_out; hp.per_round = dev_per_round;
+  hp.handoff = handoff; hp.sparse_T = sparse_T;
+  hp.launches = device_launch_counter();
+  if (!hp.launches) return PM_ERR_CUDA;
   k_ls_set_params<<<1, 1, 0, st>>>(cg.dparams, hp);
   const int blocks = (S + 255) / 256 > 0 ? (S + 255) / 256 : 1;
   k_ls_check_init<<<blocks, 256, 0, st>>>(cg.dparams);
   k_ls_check_seen<<<blocks, 256, 0, st>>>(cg.dparams);
   note_launch(3);
   PM_CUDA_TRY(cudaGetLastError());
-  PM_CUDA_TRY(cudaGraphLaunch(cg.exec, st));
-  // the graph's launches (rounds * (ncls + 1)) are counted by the caller once
-  // it has read `rounds` back
+  PM_CUDA_TRY(cudaGraphLaunch(cg.exec, st));   // its kernels count themselves on the device
   PM_CUDA_TRY(cudaFreeAsync(scratch, st));
   return PM_OK;
 }
@@ -296,19 +303,36 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   const int32_t cta_max = ls_cta_max_S();
   if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
   if (used_method) *used_method = method;
+  const int32_t sparse_T = (method == PM_LS_CLASS || method == PM_LS_WINDOW) ? ls_sparse_threshold(S, method) : 0;
+  SparseRun sr;
+  if (sparse_T > 0) {
+    const pm_status_t s = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &sr);
+    if (s != PM_OK) return s;
+  }
+  pm_status_t s;
   switch (method) {
     case PM_LS_CLASS:
-      return run_class(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+      s = run_class(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
+      break;
     case PM_LS_CTA:
       if (S > cta_max) return PM_ERR_UNSUPPORTED;
       return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     case PM_LS_WINDOW:
-      return run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+      s = run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
+      break;
     case PM_LS_PAIRWIN:
       return run_pairwin(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     default:
       return PM_ERR_UNSUPPORTED;
   }
+  if (sparse_T > 0) {
+    if (s != PM_OK) {
+      cudaFreeAsync(sr.scratch, st);
+      return s;
+    }
+    return sparse_launch(&sr, st);
+  }
+  return s;
 }
 
 // ------------------------------------------------------------ Eq. (2) ----

@@ -91,7 +91,8 @@ struct WinSmem {
 template <int K, int PPT, int MAXT>
 __global__ void __launch_bounds__(MAXT, 1)
 k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict__ Ep, int64_t ldp, int32_t S,
-            int32_t* __restrict__ perm, int32_t max_rounds, LsResult* out, int64_t* per_round, int32_t max_log) {
+            int32_t* __restrict__ perm, int32_t max_rounds, LsResult* out, int64_t* per_round, int32_t max_log,
+            int32_t* handoff, int32_t sparse_T) {
   static_assert(K % 4 == 0, "K multiple of 4");
   constexpr int KS = K + 4;
   constexpr int NP = KS / 4;       // 16-byte pieces per window
@@ -437,6 +438,10 @@ k_ls_window(const int32_t* __restrict__ E, int64_t ld, const int32_t* __restrict
     total += rs;
     if (rs == 0) break;
     if (max_rounds > 0 && rounds >= max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
+    if (handoff && rs <= sparse_T) {                   // quiet: sparse rounds take over (k_sparse.cu)
+      if (tid == 0) *handoff = 1;
+      break;
+    }
     B = 1;
     dense = rs > cl.ncls / 2;
   }
@@ -461,7 +466,7 @@ cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int6
 template <int K, int PPT, int MAXT>
 static pm_status_t launch_window_k(const int32_t* E, int64_t ldE, const int32_t* Ep, int64_t ldp, int32_t S,
                                    int32_t* perm, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
-                                   int32_t max_log, cudaStream_t st) {
+                                   int32_t max_log, cudaStream_t st, int32_t* handoff, int32_t sparse_T) {
   const size_t smem = WinSmem<K>::bytes(S);
   int dev = 0, optin = 0;
   PM_CUDA_TRY(cudaGetDevice(&dev));
@@ -473,14 +478,16 @@ static pm_status_t launch_window_k(const int32_t* E, int64_t ldE, const int32_t*
   threads = (threads + 31) / 32 * 32;
   if (threads < 32) threads = 32;
   if (threads > MAXT) return PM_ERR_UNSUPPORTED;
-  k_ls_window<K, PPT, MAXT><<<1, threads, smem, st>>>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log);
+  k_ls_window<K, PPT, MAXT><<<1, threads, smem, st>>>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log,
+                                                       handoff, sparse_T);
   note_launch();
   PM_CUDA_TRY(cudaGetLastError());
   return PM_OK;
 }
 
 pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
-                       LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
+                       LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                       int32_t* handoff, int32_t sparse_T) {
   if (S > ls_window_max_S()) return PM_ERR_UNSUPPORTED;
   const Classes cl(S);
   const int32_t m = cl.m;
@@ -498,8 +505,10 @@ pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, 
     PM_CUDA_TRY(cudaGetLastError());
   }
   pm_status_t s;
-  if (S <= 1024) s = launch_window_k<16, 1, 512>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
-  else s = launch_window_k<4, 1, 1024>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+  if (S <= 1024) s = launch_window_k<16, 1, 512>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st,
+                                                  handoff, sparse_T);
+  else s = launch_window_k<4, 1, 1024>(E, ldE, Ep, ldp, S, perm, max_rounds, dev_out, dev_per_round, max_log, st,
+                                                   handoff, sparse_T);
   PM_CUDA_TRY(cudaFreeAsync(Ep, st));
   return s;
 }

@@ -36,6 +36,38 @@ cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
   }
   return cudaMallocFromPoolAsync(p, bytes, pool, st);
 }
+
+static std::mutex g_ctr_mu;
+static unsigned long long* g_dev_ctr[64] = {};
+
+unsigned long long* device_launch_counter() {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lk(g_ctr_mu);
+  if (!g_dev_ctr[dev]) {
+    unsigned long long* p = nullptr;
+    if (cudaMalloc(&p, sizeof(unsigned long long)) != cudaSuccess) return nullptr;
+    if (cudaMemset(p, 0, sizeof(unsigned long long)) != cudaSuccess) return nullptr;
+    g_dev_ctr[dev] = p;
+  }
+  return g_dev_ctr[dev];
+}
+
+int64_t device_launch_total() {
+  int cur = 0;
+  if (cudaGetDevice(&cur) != cudaSuccess) return 0;
+  int64_t total = 0;
+  std::lock_guard<std::mutex> lk(g_ctr_mu);
+  for (int dev = 0; dev < 64; ++dev) {
+    if (!g_dev_ctr[dev]) continue;
+    unsigned long long v = 0;
+    if (cudaSetDevice(dev) == cudaSuccess &&
+        cudaMemcpy(&v, g_dev_ctr[dev], sizeof(v), cudaMemcpyDeviceToHost) == cudaSuccess)
+      total += (int64_t)v;
+  }
+  cudaSetDevice(cur);
+  return total;
+}
 }  // namespace pm
 
 using namespace pm;
@@ -89,7 +121,6 @@ pm_status_t local_search_impl(const int32_t* d_E, int64_t ld_E, int32_t S, int32
     PM_CUDA_TRY(cudaMemcpyAsync(hlog.data(), dlog, sizeof(int64_t) * hlog.size(), cudaMemcpyDeviceToHost, st));
   }
   PM_CUDA_TRY(cudaStreamSynchronize(st));
-  if (used == PM_LS_CLASS) note_launch(hres.rounds * ls_class_launches_per_round(S));
   if (h_rounds) *h_rounds = (int32_t)hres.rounds;
   if (h_swaps) *h_swaps = hres.swaps;
   if (h_per_round && len > 0)   // entries at and beyond `rounds` are zero
@@ -344,6 +375,6 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
   return PM_OK;
 }
 
-int64_t pm_launch_count(void) { return g_launches.load(); }
+int64_t pm_launch_count(void) { return g_launches.load() + device_launch_total(); }
 
 }  // extern "C"

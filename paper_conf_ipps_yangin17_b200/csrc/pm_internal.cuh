@@ -73,7 +73,8 @@ struct Classes {
       return x;
     }
     int32_t p = 2 * c + 1 - x;  // in (-m, 2m)
-    p %= m; if (p < 0) p += m;
+    if (p < 0) p += m;
+    else if (p >= m) p -= m;
     return p;
   }
 };
@@ -117,9 +118,47 @@ cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int6
 pm_status_t run_pairwin(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                         LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
-                       LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
+                       LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                       int32_t* handoff = nullptr, int32_t sparse_T = 0);
 cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm,
                         int64_t* d_cost, cudaStream_t st);
+// ---- sparse rounds (k_sparse.cu): quiet rounds of Alg. 2 ----
+struct SpParams {
+  const int32_t* E;
+  int64_t ldE;
+  int32_t* r;                  // = the caller's perm
+  int32_t* d;                  // [S] diagonal E[r[x]][x]
+  int32_t* flags;              // [ncls + 1] round stamp of classes with a pair firing at round start
+  int32_t* flist;              // [ncls + 1] stamped classes of the current round, in order
+  int32_t* gbuf;               // walk arrays when shared memory is too small (else NULL)
+  int32_t S, max_rounds, max_log;
+  int32_t pending;             // set by the dense stage when it hands over
+  int32_t use_smem;
+  int32_t nd_prev;             // slots swapped in the previous sparse round (-1: unknown)
+  int32_t* dprev;              // [S] their list
+  LsResult* out;
+  int64_t* per_round;
+  unsigned long long* launches;   // device-side launch counter (graph kernels)
+};
+struct SparseRun {
+  int32_t* pending = nullptr;  // device flag the dense stage sets
+  cudaGraphExec_t exec = nullptr;
+  int32_t* scratch = nullptr;
+};
+// Swap-count threshold at which the dense stage (WINDOW / CLASS) hands over
+// to sparse rounds; 0 = never.
+int32_t ls_sparse_threshold(int32_t S, int32_t dense_method);
+// Enqueue the parameter upload (before the dense stage) ...
+pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                           LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                           SparseRun* run);
+// ... and the sparse-round graph (after it).
+pm_status_t sparse_launch(SparseRun* run, cudaStream_t st);
+// Per-device counter of kernels launched from inside CUDA graphs (device
+// loops), added to pm_launch_count().
+unsigned long long* device_launch_counter();
+int64_t device_launch_total();
+
 // Exact min-weight perfect matching by eps-scaling auction (k_assign.cu).
 // h_stats (nullable): {bidding rounds, phases}.  Synchronises st.
 pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* perm, int64_t* price_out,

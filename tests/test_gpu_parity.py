@@ -422,3 +422,38 @@ def test_render_transposition_reproduces_target():
     I, T = pair("transposition", 512, 16)
     perm, rounds, swaps, cost, E = pm.photomosaic(dev(I), dev(T), 16)
     assert cost == 0 and (pm.render(dev(I), 16, perm).cpu().numpy() == T).all()
+
+
+# ------------------------------------------- sparse rounds (k_sparse.cu) ---
+# The dense stage (WINDOW / CLASS) hands over to exact sparse rounds after a
+# round with <= PM_LS_SPARSE_T swaps; every hand-over point must reproduce the
+# oracle bit for bit (r, rounds, swaps per round).
+@pytest.mark.parametrize("method", ["window", "class"])
+@pytest.mark.parametrize("T", ["0", "1", "40", "1000000000"])
+@pytest.mark.parametrize("shape,fam", [((128, 8, 3), "smooth"), ((512, 16, 3), "smooth"), ((90, 10, 3), "smooth"),
+                                       ((200, 5, 1), "noise"), ((128, 8, 3), "ties"), ((42, 6, 3), "transposition")])
+def test_sparse_rounds_parity(monkeypatch, method, T, shape, fam):
+    monkeypatch.setenv("PM_LS_SPARSE_T", T)
+    _check_ls(oracle_E(fam, *shape), method)
+
+
+@pytest.mark.parametrize("gmem", ["0", "1"])
+def test_sparse_rounds_global_arrays_and_resume(monkeypatch, gmem):
+    """Walk arrays in global memory (the S > 17K layout, forced), a resumed
+    search and a max_rounds cut that lands inside the sparse stage."""
+    monkeypatch.setenv("PM_LS_SPARSE_GMEM", gmem)
+    monkeypatch.setenv("PM_LS_SPARSE_T", "1000000000")
+    E_np = oracle_E("smooth", 512, 16)
+    _check_ls(E_np, "class")
+    _check_ls(E_np, "window")
+    for mr in (1, 2, 3, 5):
+        _check_ls(E_np, "window", max_rounds=mr)
+        _check_ls(E_np, "class", max_rounds=mr)
+    rng = np.random.default_rng(5)
+    _check_ls(E_np, "window", perm0=rng.permutation(E_np.shape[0]))
+
+
+def test_sparse_rounds_disabled_matches(monkeypatch):
+    monkeypatch.setenv("PM_LS_SPARSE", "0")
+    _check_ls(oracle_E("smooth", 512, 16), "window")
+    _check_ls(oracle_E("smooth", 128, 8), "class")
