@@ -9,7 +9,7 @@
 // and accumulates into an int32, and issues at the IADD3 rate (64/clk/SM,
 // tools/ubench_alu.cu).  The kernel is a register-blocked "SAD-GEMM":
 //   * CTA tile 128 (input tiles u) x 128 (target tiles v), 256 threads, each
-//     thread 8 x 8 outputs (rows ty + 16 i, cols tx + 16 j -> conflict-free
+//     thread 8 x 8 outputs (128 x 64 and 8 x 4, two CTAs per SM, for small S) (rows ty + 16 i, cols tx + 16 j -> conflict-free
 //     LDS.128 on a 80-byte padded smem row stride);
 //   * K (the P bytes of a tile) streamed in 64-byte chunks through a 4-stage
 //     cp.async.cg ring (16-byte copies, L2-only), so smem holds 16 words per
@@ -98,11 +98,12 @@ cudaError_t launch_render(const uint8_t* img, int32_t N, int32_t M, int32_t C, c
 // ---------------------------------------------------------------- Step 2 ---
 namespace sad {
 constexpr int kThreads = 256;
-constexpr int BM = 128, BN = 128;
+constexpr int BM = 128;          // tile rows (input tiles u); BN (target tiles v) is 128 or 64
 constexpr int BKW = 16;          // K words (4 bytes each) per pipeline stage
 constexpr int kStages = 4;
 constexpr int ROWW = BKW + 4;    // padded smem row stride in words (80 B)
-constexpr int kSmemBytes = kStages * (BM + BN) * ROWW * 4;   // 80 KiB
+template <int BN>
+constexpr int smem_bytes() { return kStages * (BM + BN) * ROWW * 4; }   // 80 / 60 KiB
 }  // namespace sad
 
 __device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t c) {
@@ -144,11 +145,14 @@ __device__ __forceinline__ const uint8_t* sad_tile_base(const SadGeom& geo, cons
 }
 
 // nrows rows of A (input tiles), S columns (target tiles).  kw_split: K words
-// handled by one blockIdx.z slice.
-template <bool kAtomic, bool kImage>
-__global__ void __launch_bounds__(sad::kThreads, 1)
+// handled by one blockIdx.z slice.  BN = 128: 8 x 8 outputs per thread, one
+// CTA per SM; BN = 64: 8 x 4, two CTAs per SM (for grids too small to fill
+// 148 SMs with 128 x 128 tiles without split-K).
+template <bool kAtomic, bool kImage, int BN>
+__global__ void __launch_bounds__(sad::kThreads, BN == 128 ? 1 : 2)
 k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE) {
   using namespace sad;
+  constexpr int NJ = BN / 16;                          // output columns per thread
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t* sA = smem;                                 // [kStages][BM][ROWW]
   uint32_t* sB = smem + kStages * BM * ROWW;           // [kStages][BN][ROWW]
@@ -159,44 +163,42 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
   const int32_t piece0 = blockIdx.z * kw_split / 4;    // first 16-byte piece of this K slice
   const int nkb = kw_split / BKW;
 
-  // Loader: per operand and stage, BM rows x 64 B = 512 16-byte pieces; thread
-  // tid copies pieces q = tid and q = tid + 256 (row q >> 2, part q & 3).
-  const uint8_t* baseA[2];
-  const uint8_t* baseB[2];
-  int part4[2];
-  int dst_off[2];
+  // Loader: per stage, BM (BN) rows x 64 B = 4 BM (4 BN) 16-byte pieces per
+  // operand; thread tid copies pieces q = tid + h * 256 (row q >> 2, part q & 3).
+  constexpr int HA = BM * 4 / kThreads, HB = BN * 4 / kThreads;
+  const uint8_t* baseA[HA];
+  const uint8_t* baseB[HB];
+  const int part = tid & 3;
 #pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    const int q = tid + h * kThreads;
-    const int r = q >> 2, part = q & 3;
-    int32_t ra = row0 + r; if (ra >= nrows) ra = nrows - 1;   // clamp: loaded, never stored
-    int32_t rb = col0 + r; if (rb >= S) rb = S - 1;
+  for (int h = 0; h < HA; ++h) {
+    int32_t ra = row0 + ((tid + h * kThreads) >> 2); if (ra >= nrows) ra = nrows - 1;   // clamp: loaded, never stored
     baseA[h] = sad_tile_base<kImage>(geo, geo.A, kImage ? geo.a_tile0 + ra : ra);
+  }
+#pragma unroll
+  for (int h = 0; h < HB; ++h) {
+    int32_t rb = col0 + ((tid + h * kThreads) >> 2); if (rb >= S) rb = S - 1;
     baseB[h] = sad_tile_base<kImage>(geo, geo.B, rb);
-    part4[h] = part;
-    dst_off[h] = r * ROWW + part * 4;
   }
   auto load_stage = [&](int kb, int stage) {
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int32_t p = piece0 + kb * (BKW / 4) + part4[h];
-      int64_t off;
-      if (kImage) {
-        const int32_t y = p / geo.R;
-        off = (int64_t)y * geo.rowbytes + (p - y * geo.R) * 16;
-      } else {
-        off = (int64_t)p * 16;
-      }
-      cp_async16(sA + stage * BM * ROWW + dst_off[h], baseA[h] + off);
-      cp_async16(sB + stage * BN * ROWW + dst_off[h], baseB[h] + off);
+    const int32_t p = piece0 + kb * (BKW / 4) + part;
+    int64_t off;
+    if (kImage) {
+      const int32_t y = p / geo.R;
+      off = (int64_t)y * geo.rowbytes + (p - y * geo.R) * 16;
+    } else {
+      off = (int64_t)p * 16;
     }
+#pragma unroll
+    for (int h = 0; h < HA; ++h) cp_async16(sA + stage * BM * ROWW + ((tid + h * kThreads) >> 2) * ROWW + part * 4, baseA[h] + off);
+#pragma unroll
+    for (int h = 0; h < HB; ++h) cp_async16(sB + stage * BN * ROWW + ((tid + h * kThreads) >> 2) * ROWW + part * 4, baseB[h] + off);
   };
 
-  uint32_t acc[8][8];
+  uint32_t acc[8][NJ];
 #pragma unroll
   for (int i = 0; i < 8; ++i)
 #pragma unroll
-    for (int j = 0; j < 8; ++j) acc[i][j] = 0u;
+    for (int j = 0; j < NJ; ++j) acc[i][j] = 0u;
 
 #pragma unroll
   for (int s = 0; s < kStages - 1; ++s) {
@@ -217,15 +219,15 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
     const uint32_t* b_base = sB + stage * BN * ROWW + tx * ROWW;
 #pragma unroll
     for (int kk = 0; kk < BKW; kk += 4) {
-      uint4 a[8], b[8];
+      uint4 a[8], b[NJ];
 #pragma unroll
       for (int i = 0; i < 8; ++i) a[i] = *reinterpret_cast<const uint4*>(a_base + i * 16 * ROWW + kk);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) b[j] = *reinterpret_cast<const uint4*>(b_base + j * 16 * ROWW + kk);
+      for (int j = 0; j < NJ; ++j) b[j] = *reinterpret_cast<const uint4*>(b_base + j * 16 * ROWW + kk);
 #pragma unroll
       for (int i = 0; i < 8; ++i)
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
+        for (int j = 0; j < NJ; ++j) {
           uint32_t t = acc[i][j];
           t = sad4(a[i].x, b[j].x, t);
           t = sad4(a[i].y, b[j].y, t);
@@ -243,7 +245,7 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
     if (row >= nrows) continue;
     int32_t* erow = E + (int64_t)row * ldE;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
+    for (int j = 0; j < NJ; ++j) {
       const int32_t col = col0 + tx + 16 * j;
       if (col >= S) continue;
       if (kAtomic) atomicAdd(erow + col, (int32_t)acc[i][j]);
@@ -252,26 +254,34 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
   }
 }
 
-// Host-side split-K choice: minimise waves(tiles * split) * (nkb / split) over
-// the divisors of nkb that leave >= 2 K-chunks per CTA.
-static int choose_split(int64_t tiles, int nkb, int sms) {
-  int best = 1;
+// Host-side tiling choice: 128 x 128 tiles with split-K over the divisors of
+// nkb, or 128 x 64 tiles (two CTAs per SM, half the work per tile) without
+// split-K.  Cost = waves * per-CTA work, with a small bias against split-K
+// (its memset and atomics).
+struct SadPlan { int bn, split; };
+static SadPlan choose_plan(int64_t nrows, int64_t S, int nkb, int sms) {
+  SadPlan best{128, 1};
   double best_cost = 1e300;
+  const int64_t gy = (nrows + sad::BM - 1) / sad::BM;
   for (int s = 1; s <= nkb; ++s) {
     if (nkb % s) continue;
     if (s > 1 && nkb / s < 2) break;
-    const int64_t ctas = tiles * s;
-    const int64_t waves = (ctas + sms - 1) / sms;
-    // small bias against splitting (memset + atomics)
-    const double cost = (double)waves * (nkb / s) * (s > 1 ? 1.03 : 1.0);
-    if (cost < best_cost - 1e-9) { best_cost = cost; best = s; }
+    const int64_t ctas = gy * ((S + 127) / 128) * s;
+    const double cost = (double)((ctas + sms - 1) / sms) * (nkb / s) * (s > 1 ? 1.10 : 1.0);
+    if (cost < best_cost - 1e-9) { best_cost = cost; best = {128, s}; }
+  }
+  {
+    const int64_t ctas = gy * ((S + 63) / 64);
+    const double cost = (double)((ctas + sms - 1) / sms) * nkb * 0.5;   // half-size tiles (two per SM hide latency)
+    if (cost < best_cost - 1e-9) { best_cost = cost; best = {64, 1}; }
   }
   return best;
 }
 
-template <bool kAtomic, bool kImage>
+template <bool kAtomic, bool kImage, int BN>
 static cudaError_t sad_set_attr() {
-  return cudaFuncSetAttribute(k_sad<kAtomic, kImage>, cudaFuncAttributeMaxDynamicSharedMemorySize, sad::kSmemBytes);
+  return cudaFuncSetAttribute(k_sad<kAtomic, kImage, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              sad::smem_bytes<BN>());
 }
 
 static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows, int32_t S, int32_t P,
@@ -284,29 +294,39 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
   static std::atomic<uint64_t> attr_done{0};   // one bit per device ordinal
   if (dev < 64 && !(attr_done.load() & (1ull << dev))) {
     cudaError_t e;
-    if ((e = sad_set_attr<false, false>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<true, false>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<false, true>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<true, true>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<false, false, 128>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<true, false, 128>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<false, true, 128>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<true, true, 128>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<false, false, 64>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<false, true, 64>()) != cudaSuccess) return e;
     attr_done.fetch_or(1ull << dev);
   }
   const int kw = image ? P / 4 : (int)(geo.ldt / 4);
   const int nkb = kw / BKW;
-  const int64_t gx = (S + BN - 1) / BN, gy = (nrows + BM - 1) / BM;
+  const int64_t gy = (nrows + BM - 1) / BM;
   if (gy > 65535) return cudaErrorInvalidValue;
-  const int split = choose_split(gx * gy, nkb, sms);
-  dim3 grid((unsigned)gx, (unsigned)gy, (unsigned)split);
+  const SadPlan plan = choose_plan(nrows, S, nkb, sms);
+  if (plan.bn == 64) {
+    dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, 1);
+    if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
+    else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
+    note_launch();
+    return cudaGetLastError();
+  }
+  const int split = plan.split;
+  dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
   if (split > 1) {
     // split-K accumulates with red.add: zero the [nrows][S] window of E first
     cudaError_t e = (ldE == S)
         ? cudaMemsetAsync(E, 0, sizeof(int32_t) * (size_t)nrows * S, st)
         : cudaMemset2DAsync(E, sizeof(int32_t) * ldE, 0, sizeof(int32_t) * S, nrows, st);
     if (e != cudaSuccess) return e;
-    if (image) k_sad<true, true><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw / split, E, ldE);
-    else k_sad<true, false><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw / split, E, ldE);
+    if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE);
+    else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE);
   } else {
-    if (image) k_sad<false, true><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw, E, ldE);
-    else k_sad<false, false><<<grid, kThreads, kSmemBytes, st>>>(geo, nrows, S, kw, E, ldE);
+    if (image) k_sad<false, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE);
+    else k_sad<false, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE);
   }
   note_launch();
   return cudaGetLastError();
