@@ -52,11 +52,17 @@ typedef enum {
                           from L2/HBM (S <= pm_ls_cta_max_S())                */
   PM_LS_WINDOW = 3,    /* one CTA, plus a shared-memory window of each slot's
                           upcoming E entries streamed ahead of the classes    */
-  PM_LS_PAIRWIN = 4    /* per round: a grid-wide kernel tabulates every pair's
+  PM_LS_PAIRWIN = 4,   /* per round: a grid-wide kernel tabulates every pair's
                           two terms of line 5 at the round's start, one CTA
                           streams the class rows and patches swapped slots;
                           rounds looped on the device (CUDA-graph WHILE node);
                           40 <= S <= 2048 on this build                       */
+  PM_LS_WALK = 5       /* every round as a sparse round: a whole-GPU test of
+                          every pair on the round's start state marks the
+                          classes that can fire, then a thread-block cluster
+                          walks the classes in order, testing only those
+                          classes and the pairs of already-swapped slots;
+                          rounds looped on the device (CUDA-graph WHILE node) */
 } pm_ls_method_t;
 
 const char* pm_status_string(pm_status_t s);

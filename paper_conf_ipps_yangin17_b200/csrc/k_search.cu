@@ -320,6 +320,15 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
     case PM_LS_WINDOW:
       s = run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
       break;
+    case PM_LS_WALK: {
+      // every round a sparse round: start-state scan + cluster walk (S >= 2)
+      if (S < 2) return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+      PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
+      SparseRun wr;
+      const pm_status_t s0 = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &wr, 1);
+      if (s0 != PM_OK) return s0;
+      return sparse_launch(&wr, st);
+    }
     case PM_LS_PAIRWIN:
       return run_pairwin(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     default:

@@ -449,7 +449,7 @@ struct SpGraph {
 };
 
 static std::mutex g_sp_mu;
-static std::map<std::tuple<int, int32_t, cudaStream_t, bool>, SpGraph> g_sp_graphs;
+static std::map<std::tuple<int, int32_t, cudaStream_t, bool, bool>, SpGraph> g_sp_graphs;
 
 static int scan_blocks(int32_t S) {
   const int64_t total = (int64_t)Classes(S).ncls * Classes(S).npairs;
@@ -458,7 +458,7 @@ static int scan_blocks(int32_t S) {
   return b < 1 ? 1 : (int)b;
 }
 
-static cudaError_t build_sparse_graph(int32_t S, bool use_smem, SpGraph& out) {
+static cudaError_t build_sparse_graph(int32_t S, bool use_smem, bool cluster, SpGraph& out) {
   cudaError_t e = cudaMalloc(&out.dparams, sizeof(SpParams));
   if (e != cudaSuccess) return e;
   cudaGraph_t g = nullptr;
@@ -466,7 +466,7 @@ static cudaError_t build_sparse_graph(int32_t S, bool use_smem, SpGraph& out) {
   cudaGraphConditionalHandle h;
   if ((e = cudaGraphConditionalHandleCreate(&h, g, 0, cudaGraphCondAssignDefault)) != cudaSuccess) return e;
   const size_t smem = use_smem ? walk_smem_bytes(S) : 0;
-  if (use_smem &&
+  if (use_smem && !cluster &&
       (e = cudaFuncSetAttribute(k_sp_walk<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
     return e;
   // [begin] -> while { scan ; walk }
@@ -493,8 +493,17 @@ static cudaError_t build_sparse_graph(int32_t S, bool use_smem, SpGraph& out) {
   if ((e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed)) != cudaSuccess)
     return e;
   k_sp_scan<<<scan_blocks(S), 256, 0, cs>>>(out.dparams);
-  if (use_smem) k_sp_walk<true><<<1, kWalkThreads, smem, cs>>>(out.dparams, h);
-  else k_sp_walk<false><<<1, kWalkThreads, 0, cs>>>(out.dparams, h);
+  if (cluster) {
+    if ((e = launch_cwalk(out.dparams, h, S, use_smem, cs)) != cudaSuccess) {
+      cudaStreamEndCapture(cs, &captured);
+      cudaStreamDestroy(cs);
+      return e;
+    }
+  } else if (use_smem) {
+    k_sp_walk<true><<<1, kWalkThreads, smem, cs>>>(out.dparams, h);
+  } else {
+    k_sp_walk<false><<<1, kWalkThreads, 0, cs>>>(out.dparams, h);
+  }
   captured = body;
   e = cudaStreamEndCapture(cs, &captured);
   cudaStreamDestroy(cs);
@@ -513,37 +522,48 @@ int32_t ls_sparse_threshold(int32_t S, int32_t dense_method) {
   if (S < 2 || !env_or("PM_LS_SPARSE", 1)) return 0;
   const int32_t t = env_or("PM_LS_SPARSE_T", -1);
   if (t >= 0) return t;
-  // measured (profiles/r01_profile.md): a sparse round costs ~2 windows of
-  // ~1.3 us per swap it performs plus ~15 us fixed, a WINDOW round ~0.3 us
-  // per class and a CLASS round ~2.3 us per class; with swaps falling ~3x per
-  // round this puts the hand-over at ~S^2/1024 swaps (S = 256: 64, 1024: 1024)
+  // measured on B200: S <= 2048 (WINDOW + one-CTA walk): a
+  // sparse round costs ~2 windows of ~1.3 us per swap plus ~15 us, a WINDOW
+  // round ~0.3 us per class; with swaps falling ~3x per round the hand-over
+  // sits at ~S^2/1024 swaps (S = 256: 64, 1024: 1024).  S > 2048 (CLASS +
+  // cluster walk): the walk's windows are gather-bound once the dirty set
+  // holds ~S slots, so hand over below ~3S/4 swaps (S = 4096: after the
+  // 2489-swap round, 27 vs 33 ms; S = 16384: after the 4715-swap round,
+  // 240 vs 375 ms at S^2/1024).
   (void)dense_method;
+  if (S > 2048) return (int32_t)((int64_t)S * 3 / 4);
   const int64_t t2 = (int64_t)S * S / 1024;
   return (int32_t)(t2 < 1 ? 1 : (t2 > INT32_MAX ? INT32_MAX : t2));
 }
 
 pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                            LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                           SparseRun* run) {
+                           SparseRun* run, int32_t pending0) {
   int dev = 0, optin = 0;
   PM_CUDA_TRY(cudaGetDevice(&dev));
   PM_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
-  const bool use_smem = walk_smem_bytes(S) + 1024 <= (size_t)optin && !env_or("PM_LS_SPARSE_GMEM", 0);
+  // the walk: one CTA for S <= 2048, a thread-block cluster (k_cwalk.cu)
+  // beyond (measured: its cluster barrier per window only pays once the dirty
+  // sets outgrow one CTA); PM_LS_CWALK=0/1 forces either
+  const int32_t cw_env = env_or("PM_LS_CWALK", -1);
+  const bool cluster = cw_env < 0 ? S > 2048 : cw_env != 0;
+  const bool use_smem = (cluster ? cwalk_smem_ok(S, optin) : walk_smem_bytes(S) + 1024 <= (size_t)optin) &&
+                        !env_or("PM_LS_SPARSE_GMEM", 0);
   SpGraph sg;
   {
     std::lock_guard<std::mutex> lk(g_sp_mu);
-    auto key = std::make_tuple(dev, S, st, use_smem);
+    auto key = std::make_tuple(dev, S, st, use_smem, cluster);
     auto it = g_sp_graphs.find(key);
     if (it == g_sp_graphs.end()) {
       SpGraph ng;
-      PM_CUDA_TRY(build_sparse_graph(S, use_smem, ng));
+      PM_CUDA_TRY(build_sparse_graph(S, use_smem, cluster, ng));
       it = g_sp_graphs.emplace(key, ng).first;
     }
     sg = it->second;
   }
   const Classes cl(S);
-  const size_t words = (size_t)S * 2 /*d, dprev*/ + (size_t)(cl.ncls + 1) * 2 /*flags, flist*/ +
-                       (use_smem ? 0 : (size_t)S * 4) /*R, D, L, dirty*/;
+  const size_t gwords = use_smem ? 0 : (cluster ? cwalk_gbuf_bytes(S) / 4 : (size_t)S * 4);   // R, D, L, dirty
+  const size_t words = (size_t)S * 2 /*d, dprev*/ + (size_t)(cl.ncls + 1) * 2 /*flags, flist*/ + gwords;
   int32_t* scratch = nullptr;
   PM_CUDA_TRY(pm::scratch_alloc(&scratch, sizeof(int32_t) * words, st));
   PM_CUDA_TRY(cudaMemsetAsync(scratch + S, 0, sizeof(int32_t) * (size_t)(cl.ncls + 1), st));
@@ -556,7 +576,7 @@ pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* pe
   hp.gbuf = use_smem ? nullptr : hp.dprev + S;
   hp.nd_prev = -1;
   hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
-  hp.pending = 0; hp.use_smem = use_smem ? 1 : 0;
+  hp.pending = pending0; hp.use_smem = use_smem ? 1 : 0;
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.launches = device_launch_counter();
   if (!hp.launches) return PM_ERR_CUDA;
@@ -567,6 +587,31 @@ pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* pe
   run->exec = sg.exec;
   run->scratch = scratch;
   return PM_OK;
+}
+
+__global__ void k_perm_count(const int32_t* __restrict__ perm, int32_t S, int32_t* __restrict__ seen, LsResult* out) {
+  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x) {
+    const int32_t t = perm[u];
+    if (t < 0 || t >= S) out->status = PM_ERR_NOT_PERMUTATION;
+    else atomicAdd(seen + t, 1);
+  }
+}
+__global__ void k_perm_seen(const int32_t* __restrict__ seen, int32_t S, LsResult* out) {
+  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x)
+    if (seen[u] != 1) out->status = PM_ERR_NOT_PERMUTATION;
+}
+
+cudaError_t launch_perm_check(const int32_t* perm, int32_t S, LsResult* dev_out, cudaStream_t st) {
+  int32_t* seen = nullptr;
+  cudaError_t e = pm::scratch_alloc(&seen, sizeof(int32_t) * (size_t)S, st);
+  if (e != cudaSuccess) return e;
+  if ((e = cudaMemsetAsync(seen, 0, sizeof(int32_t) * (size_t)S, st)) != cudaSuccess) return e;
+  const int blocks = (S + 255) / 256 < 1184 ? (S + 255) / 256 : 1184;
+  k_perm_count<<<blocks, 256, 0, st>>>(perm, S, seen, dev_out);
+  k_perm_seen<<<blocks, 256, 0, st>>>(seen, S, dev_out);
+  note_launch(2);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  return cudaFreeAsync(seen, st);
 }
 
 pm_status_t sparse_launch(SparseRun* run, cudaStream_t st) {

@@ -145,13 +145,21 @@ struct SparseRun {
   cudaGraphExec_t exec = nullptr;
   int32_t* scratch = nullptr;
 };
+// The walk on a thread-block cluster (k_cwalk.cu).
+bool cwalk_smem_ok(int32_t S, int optin);
+size_t cwalk_gbuf_bytes(int32_t S);
+cudaError_t launch_cwalk(SpParams* p, cudaGraphConditionalHandle h, int32_t S, bool smem, cudaStream_t st);
 // Swap-count threshold at which the dense stage (WINDOW / CLASS) hands over
 // to sparse rounds; 0 = never.
 int32_t ls_sparse_threshold(int32_t S, int32_t dense_method);
 // Enqueue the parameter upload (before the dense stage) ...
+// pending0 = 1 runs every round as a sparse round (PM_LS_WALK); the caller
+// has checked that perm is a bijection.
 pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                            LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                           SparseRun* run);
+                           SparseRun* run, int32_t pending0 = 0);
+// dev_out->status = PM_ERR_NOT_PERMUTATION unless perm is a bijection of [0, S).
+cudaError_t launch_perm_check(const int32_t* perm, int32_t S, LsResult* dev_out, cudaStream_t st);
 // ... and the sparse-round graph (after it).
 pm_status_t sparse_launch(SparseRun* run, cudaStream_t st);
 // Per-device counter of kernels launched from inside CUDA graphs (device

@@ -20,7 +20,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libpm.so")
 
 PM_OK, PM_ERR_INVALID, PM_ERR_CUDA, PM_ERR_NOT_CONVERGED, PM_ERR_UNSUPPORTED, PM_ERR_NOT_PERMUTATION = range(6)
-METHODS = {"auto": 0, "class": 1, "cta": 2, "window": 3, "pairwin": 4}
+METHODS = {"auto": 0, "class": 1, "cta": 2, "window": 3, "pairwin": 4, "walk": 5}
 
 _lib = None
 _P = ctypes.c_void_p

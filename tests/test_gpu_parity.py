@@ -150,39 +150,39 @@ def _check_ls(E_np, method, perm0=None, max_rounds=0):
     return ref
 
 
-@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "shuffle", "transposition", "identical"])
 def test_local_search_parity_config1(method, fam):
     _check_ls(oracle_E(fam, 128, 8), method)
 
 
-@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
 def test_local_search_parity_config2(method, fam):
     _check_ls(oracle_E(fam, 512, 16), method)
 
 
-@pytest.mark.parametrize("method", ["auto", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "walk", "cta", "class"])
 def test_local_search_parity_config3(method):
     ref = _check_ls(oracle_E("smooth", 1024, 16), method)
     assert ref[1] >= 3
 
 
-@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("N,M,C", [(90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (30, 10, 3), (64, 64, 1)])
 def test_local_search_parity_ragged_and_odd(method, N, M, C):
     # S = 81, 49, 9 are odd (the fixed point idles, reading R9); S = 1 trivial
     _check_ls(oracle_E("smooth", N, M, C), method)
 
 
-@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
 def test_local_search_resume_from_any_bijection(method):
     E = oracle_E("noise", 128, 8)
     rng = np.random.default_rng(3)
     _check_ls(E, method, perm0=rng.permutation(256).astype(np.int32))
 
 
-@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
 def test_local_search_max_rounds_then_resume(method):
     E_np = oracle_E("smooth", 512, 16)
     ref = _check_ls(E_np, method, max_rounds=2)
@@ -190,7 +190,7 @@ def test_local_search_max_rounds_then_resume(method):
     _check_ls(E_np, method, perm0=ref[0])
 
 
-@pytest.mark.parametrize("method", ["pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
 def test_local_search_rejects_non_permutation(method):
     E = dev(oracle_E("smooth", 128, 8))
     bad = torch.arange(256, dtype=torch.int32, device=DEV)
@@ -210,7 +210,7 @@ def test_local_search_random_small_matrices():
     for _ in range(25):
         S = int(rng.integers(1, 10))
         E = rng.integers(0, 4, size=(S, S)).astype(np.int32)
-        for method in ("window", "cta", "class"):
+        for method in ("walk", "window", "cta", "class"):
             _check_ls(E, method)
         if S >= 40:
             _check_ls(E, "pairwin")
@@ -428,22 +428,29 @@ def test_render_transposition_reproduces_target():
 # The dense stage (WINDOW / CLASS) hands over to exact sparse rounds after a
 # round with <= PM_LS_SPARSE_T swaps; every hand-over point must reproduce the
 # oracle bit for bit (r, rounds, swaps per round).
+@pytest.mark.parametrize("cwalk", ["0", "1"])
 @pytest.mark.parametrize("method", ["window", "class"])
 @pytest.mark.parametrize("T", ["0", "1", "40", "1000000000"])
 @pytest.mark.parametrize("shape,fam", [((128, 8, 3), "smooth"), ((512, 16, 3), "smooth"), ((90, 10, 3), "smooth"),
                                        ((200, 5, 1), "noise"), ((128, 8, 3), "ties"), ((42, 6, 3), "transposition")])
-def test_sparse_rounds_parity(monkeypatch, method, T, shape, fam):
+def test_sparse_rounds_parity(monkeypatch, cwalk, method, T, shape, fam):
+    monkeypatch.setenv("PM_LS_CWALK", cwalk)
     monkeypatch.setenv("PM_LS_SPARSE_T", T)
     _check_ls(oracle_E(fam, *shape), method)
 
 
+@pytest.mark.parametrize("cwalk", ["0", "1"])
 @pytest.mark.parametrize("gmem", ["0", "1"])
-def test_sparse_rounds_global_arrays_and_resume(monkeypatch, gmem):
+def test_sparse_rounds_global_arrays_and_resume(monkeypatch, gmem, cwalk):
     """Walk arrays in global memory (the S > 17K layout, forced), a resumed
     search and a max_rounds cut that lands inside the sparse stage."""
     monkeypatch.setenv("PM_LS_SPARSE_GMEM", gmem)
+    monkeypatch.setenv("PM_LS_CWALK", cwalk)
     monkeypatch.setenv("PM_LS_SPARSE_T", "1000000000")
     E_np = oracle_E("smooth", 512, 16)
+    _check_ls(E_np, "walk")
+    for mr in (1, 2, 4):
+        _check_ls(E_np, "walk", max_rounds=mr)
     _check_ls(E_np, "class")
     _check_ls(E_np, "window")
     for mr in (1, 2, 3, 5):
@@ -457,3 +464,29 @@ def test_sparse_rounds_disabled_matches(monkeypatch):
     monkeypatch.setenv("PM_LS_SPARSE", "0")
     _check_ls(oracle_E("smooth", 512, 16), "window")
     _check_ls(oracle_E("smooth", 128, 8), "class")
+
+
+# ---------------------------------- cluster walk (k_cwalk.cu), all rounds ---
+@pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "transposition", "identical", "shuffle"])
+@pytest.mark.parametrize("N,M,C", [(128, 8, 3), (512, 16, 3), (90, 10, 3), (200, 5, 1), (1152, 32, 1), (1440, 32, 1)])
+def test_walk_all_rounds_parity(fam, N, M, C):
+    # S = 256, 1024, 81 (odd), 1600, 1296, 2025 (odd): every round as scan + cluster walk
+    _check_ls(oracle_E(fam, N, M, C), "walk")
+
+
+def test_walk_mailbox_overflow_falls_back_exactly():
+    # T = I with the tiles of 63 pairs of the first colour class exchanged: from
+    # the identity all 63 fire in that class, more than one CTA's mailbox holds
+    # (k_cwalk.cu), so every CTA re-tests the class in full
+    I, _ = pair("smooth", 512, 16)
+    g, M = 32, 16
+    groups = oracle.edge_coloring(g * g)          # [class][pair][2]
+    Tt = I.copy()
+    for a, b in groups[0][:63]:
+        ya, xa, yb, xb = (a // g) * M, (a % g) * M, (b // g) * M, (b % g) * M
+        ta = Tt[ya:ya + M, xa:xa + M].copy()
+        Tt[ya:ya + M, xa:xa + M] = Tt[yb:yb + M, xb:xb + M]
+        Tt[yb:yb + M, xb:xb + M] = ta
+    E_np = oracle.error_matrix(I, Tt, M)
+    ref = _check_ls(E_np, "walk")
+    assert ref[3][0] >= 63
