@@ -57,12 +57,20 @@ typedef enum {
                           streams the class rows and patches swapped slots;
                           rounds looped on the device (CUDA-graph WHILE node);
                           40 <= S <= 2048 on this build                       */
-  PM_LS_WALK = 5       /* every round as a sparse round: a whole-GPU test of
+  PM_LS_WALK = 5,      /* every round as a sparse round: a whole-GPU test of
                           every pair on the round's start state marks the
                           classes that can fire, then a thread-block cluster
                           walks the classes in order, testing only those
                           classes and the pairs of already-swapped slots;
                           rounds looped on the device (CUDA-graph WHILE node) */
+  PM_LS_TRAP = 6       /* whole GPU, temporal blocking of the class sequence:
+                          pair k of class c+1 depends only on pairs k-1..k+1
+                          of class c, so a warp replays T classes on the
+                          slots of pairs [k0-T, k1+T) in shared memory (E
+                          entries staged as per-tile stride-2 runs) and
+                          writes back pairs [k0, k1); one grid barrier per
+                          T classes (persistent cooperative kernel); even
+                          S >= 256                                            */
 } pm_ls_method_t;
 
 const char* pm_status_string(pm_status_t s);
@@ -242,6 +250,11 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
  * launched, which count themselves on the device -- so this call reads a
  * device counter back and synchronises with the devices it has used. */
 int64_t pm_launch_count(void);
+
+/* Test hook: E lookups PM_LS_TRAP had to serve from global memory because
+ * they fell outside the staged runs (expected 0; the result is exact either
+ * way) since the last call.  Synchronises the current device; -1 on error. */
+int64_t pm_debug_trap_misses(void);
 
 #ifdef __cplusplus
 }

@@ -303,7 +303,9 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   const int32_t cta_max = ls_cta_max_S();
   if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
   if (used_method) *used_method = method;
-  const int32_t sparse_T = (method == PM_LS_CLASS || method == PM_LS_WINDOW) ? ls_sparse_threshold(S, method) : 0;
+  if (method == PM_LS_TRAP && (S < ls_trap_min_S() || (S & 1))) return PM_ERR_UNSUPPORTED;
+  const int32_t sparse_T = (method == PM_LS_CLASS || method == PM_LS_WINDOW || method == PM_LS_TRAP)
+                               ? ls_sparse_threshold(S, method) : 0;
   SparseRun sr;
   if (sparse_T > 0) {
     const pm_status_t s = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &sr);
@@ -317,6 +319,9 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
     case PM_LS_CTA:
       if (S > cta_max) return PM_ERR_UNSUPPORTED;
       return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+    case PM_LS_TRAP:
+      s = run_trap(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
+      break;
     case PM_LS_WINDOW:
       s = run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
       break;

@@ -1,0 +1,442 @@
+// k_trap.cu -- Algorithm 2 on the whole GPU by temporal blocking
+// of the colour-class sequence (method PM_LS_TRAP).
+//
+// Structure used.  Class c pairs slot u0+k with u0-k (mod m), k = 1..K, and
+// u0 with S-1 (k = 0), where u0 = c + (m+1)/2 and K = S/2 - 1 (Theorem 1,
+// P:139; R8).  From class c to c+1, u0 advances by one, so the two slots of
+// pair k at class c+1 are the first slot of pair k+1 and the second slot of
+// pair k-1 at class c (the ends reflect: pair 0 keeps S-1, pair K takes its
+// own second slot).  The state of pair k after class c+1 therefore depends on
+// pairs k-1..k+1 after class c only: a 1-D three-point stencil in k over the
+// class index.  Alg. 2's exact result for the pairs [k0, k1) after T more
+// classes is a function of the state of pairs [k0-T, k1+T) alone.
+//
+// Kernel.  One persistent cooperative grid.  A phase covers T consecutive
+// classes of a round.  The pairs are cut into chunks of W owned pairs; a warp
+// takes a chunk, copies the state (r, d) of the slots of its extended range
+// [k0-T, k1+T) into shared memory, replays the T classes on it (the valid
+// range shrinks by one pair per side and class, "overlapped tiling") and
+// writes back the slots of its owned pairs.  Phases are separated by a grid
+// barrier, state ping-pongs between two global buffers.  Each pair test is
+// line 5 with two entries carried in d (as every other method here):
+// d[u] + d[v] > E[r[v]][u] + E[r[u]][v], strict (R6).
+//
+// E entries a chunk can need.  A tile starting at slot s0 whose class-c0
+// partner is p0 only ever sits at, or is tested against, slots s0 + 2j and
+// p0 + 2j (j < T) while it stays away from pair 0: the partner of slot x in
+// class c is 2c+1-x.  Through pair 0 (chunks with k0 <= T) it can also meet
+// u0 .. u0+2T and S-1.  So each tile of the chunk gets two stride-2 runs of T
+// entries of its E row, E[t][S-1], and for the first chunk(s) the contiguous
+// run E[t][u0 .. u0+2T]: O(T) entries per tile instead of the O(W+2T) of a
+// full sub-block.  A lookup outside the runs (never expected) falls back to a
+// global load and is counted (pm_debug_trap_misses), so the result is exact
+// regardless.
+#include <cuda_runtime.h>
+
+#include <cstdlib>
+
+#include "pm_internal.cuh"
+
+namespace pm {
+
+__device__ unsigned long long g_trap_misses;
+
+struct TrapParams {
+  const int32_t* E;
+  int64_t ldE;
+  int32_t* rbuf[2];            // rbuf[0] = the caller's perm
+  int32_t* dbuf[2];
+  int32_t S, max_rounds, max_log, sparse_T;
+  int32_t W, nchunks;
+  int32_t gsz;                 // warps per chunk group
+  int32_t prof;                // PM_TRAP_PROF: block 0 thread 0 phase timers -> per_round[192..195]
+  unsigned int* bar;           // grid barrier counter (zeroed before launch)
+  unsigned long long* rsw;     // [3] swaps per round, rotating
+  LsResult* out;
+  int64_t* per_round;
+  int32_t* handoff;
+  unsigned long long* launches;
+};
+
+template <int PPL, int T>
+struct TrapSmem {
+  static constexpr int X = 32 * PPL;        // pairs of an extended range
+  static constexpr int L = 2 * X;           // slots (= tiles) of an extended range
+  // staged row of local tile i: run0 [R0, R0+T+1) = E[g][p0 + 2j], run1
+  // [R1, R1+T+1) = E[g][s0 + 2j], E[g][S-1] at CL, runU [RU, RU+2T+2) =
+  // E[g][u0 + z] (pair-0 light cone only); odd stride (banks)
+  static constexpr int R0 = 0, R1 = T + 1, CL = 2 * T + 2, RU = 2 * T + 3;
+  static constexpr int NE = 2 * T + 3;      // entries staged for every tile
+  static constexpr int NU = 2 * T + 2;      // runU entries
+  static constexpr int RS = 4 * T + 5;
+  static constexpr int ints = L * (4 + 1 + RS);   // int4 state + g + rows
+  static constexpr size_t bytes = sizeof(int32_t) * (size_t)ints;
+};
+
+__device__ __forceinline__ int32_t wrap_m(int32_t x, int32_t m) {
+  x = x < 0 ? x + m : x;
+  return x >= m ? x - m : x;
+}
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ void cp_async4(int32_t* dst, const int32_t* src) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(s), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+// Barrier of the nthr threads of one chunk group (named barrier id >= 1).
+__device__ __forceinline__ void group_sync(int id, int nthr) {
+  if (nthr == 32) __syncwarp();
+  else asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthr) : "memory");
+}
+
+__device__ __forceinline__ void grid_barrier(unsigned int* bar, unsigned int target) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
+    unsigned int v;
+    do {
+      asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(bar) : "memory");
+    } while (v < target);
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+  }
+  __syncthreads();
+}
+
+// Local slot j of a chunk's extended range [a, b): j < nA -> slot u0 + a + j
+// (first slots), j < nA + nB -> slot u0 - (a2 + j - nA) (second slots),
+// j = nA + nB -> S - 1 (only when a == 0).  Pair k at step t (class c0 + t)
+// has slots u0 + t + k and u0 + t - k (or S - 1 for k = 0).
+struct TrapChunk {
+  int32_t a, b, a2, nA, nB, Lc, K, m;
+  __device__ __forceinline__ void local_slots(int32_t t, int32_t k, int32_t& j1, int32_t& j2) const {
+    const int32_t o1 = t + k;
+    j1 = (o1 <= K) ? o1 - a : nA + (m - o1 - a2);
+    const int32_t o2 = t - k;
+    j2 = (k == 0) ? Lc - 1 : ((o2 >= 0) ? o2 - a : nA + (k - t - a2));
+  }
+  __device__ __forceinline__ int32_t slot_of(int32_t j, int32_t u0, int32_t S) const {
+    if (j < nA) return wrap_m(u0 + a + j, m);
+    if (j < nA + nB) return wrap_m(u0 - (a2 + j - nA), m);
+    return S - 1;
+  }
+};
+
+// State of a slot: {tile | inc << 16, d, pp, po}: pp indexes the staged
+// E[tile][partner of the slot in the current class], po the staged
+// E[tile][slot + 2].  The partner of slot y in class c is 2c+1-y (mod m), so
+// while a tile stays its partner advances by 2 (pp += inc: consecutive
+// entries of a stride-2 run, inc = 1, or of runU, inc = 2) and after a swap
+// its new partner is its old slot + 2 (pp <- po, po <- pp + inc).  The slot
+// S-1 (pair 0) walks u0, u0+1, ... through runU with inc = 1.
+template <int PPL, int T>
+__global__ void __launch_bounds__(256, 1)
+k_ls_trap(const TrapParams p) {
+  using SM = TrapSmem<PPL, T>;
+  constexpr int L = SM::L, RS = SM::RS, X = SM::X;
+  extern __shared__ __align__(16) int32_t sm[];
+  const int gsz = p.gsz;                       // warps per chunk group
+  const int cpc = (blockDim.x >> 5) / gsz;     // chunk groups per CTA
+  const int grp = (threadIdx.x >> 5) / gsz;
+  const int GT = 32 * gsz;
+  const int gt = threadIdx.x - grp * GT;
+  int32_t* ws = sm + (size_t)grp * SM::ints;
+  int4* s_st = reinterpret_cast<int4*>(ws);
+  int32_t* s_g = ws + 4 * L;
+  int32_t* s_E = s_g + L;
+  __shared__ int32_t s_cta_sw;
+  __shared__ unsigned long long s_rs;
+
+  const int32_t* __restrict__ E = p.E;
+  const int64_t ld = p.ldE;
+  const int32_t S = p.S;
+  const Classes cl(S);
+  const int32_t m = cl.m, H = cl.half, K = cl.npairs - 1, ncls = cl.ncls;
+  const int32_t W = p.W;
+  const unsigned nblk = gridDim.x;
+  unsigned int bar_target = 0;
+  const int ngrp_tot = nblk * cpc;
+  const int gid = blockIdx.x * cpc + grp;
+
+  if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.launches, 1ull);
+  if (p.out->status != PM_OK) return;   // grid-uniform (written before launch)
+
+  if (threadIdx.x == 0) s_cta_sw = 0;
+  // d[x] = E[r[x]][x] (the maintained diagonal)
+  for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
+    __stcg(p.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(p.rbuf[0] + x) * ld + x));
+  bar_target += nblk;
+  grid_barrier(p.bar, bar_target);
+
+  int cur = 0;
+  int32_t rounds = 0;
+  int64_t total = 0;
+  int status = PM_OK;
+  const bool prof = p.prof && blockIdx.x == 0 && threadIdx.x == 0 && p.max_log >= 200;
+  unsigned long long t_ld = 0, t_st = 0, t_bar = 0, n_ph = 0, tq = prof ? gtimer() : 0;
+  const int npass = (p.nchunks + ngrp_tot - 1) / ngrp_tot;
+  for (;;) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
+    for (int32_t c0 = 0; c0 < ncls; c0 += T) {
+      const int32_t Tp = min(T, ncls - c0);
+      const int32_t u0 = wrap_m(c0 + H, m);
+      const int32_t* __restrict__ rc = cur ? p.rbuf[1] : p.rbuf[0];
+      const int32_t* __restrict__ dc = cur ? p.dbuf[1] : p.dbuf[0];
+      int32_t* rn = cur ? p.rbuf[0] : p.rbuf[1];
+      int32_t* dn = cur ? p.dbuf[0] : p.dbuf[1];
+      int mysw = 0;
+      for (int pass = 0; pass < npass; ++pass) {
+        const int32_t ch = gid + pass * ngrp_tot;
+        const bool have = ch < p.nchunks;
+        TrapChunk C;
+        const int32_t k0 = ch * W, k1 = min(k0 + W, K + 1);
+        C.a = max(k0 - Tp, 0); C.b = min(k1 + Tp, K + 1);
+        C.a2 = max(C.a, 1);
+        C.nA = C.b - C.a; C.nB = C.b - C.a2;
+        const bool low = (C.a == 0);
+        C.Lc = C.nA + C.nB + (low ? 1 : 0);
+        C.K = K; C.m = m;
+        const int32_t Lc = C.Lc;
+        if (have) {
+          // ---- one thread per local slot j (= local tile j): its state, then
+          // its tile's E row pieces, every copy independent of the others ----
+          for (int32_t j = gt; j < Lc; j += GT) {
+            const int32_t x = C.slot_of(j, u0, S);
+            const int32_t g = __ldcg(rc + x);
+            const int32_t d = __ldcg(dc + x);
+            s_g[j] = g;
+            const bool fx = (x == S - 1);
+            s_st[j] = fx ? make_int4(j | (1 << 16), d, j * RS + SM::RU, 0)
+                         : make_int4(j | (1 << 16), d, j * RS + SM::R0, j * RS + SM::R1 + 1);
+            const int32_t* row = E + (int64_t)g * ld;
+            int32_t* dst = s_E + j * RS;
+            // run0: E[g][p0 + 2c], run1: E[g][x + 2c] (c <= T), E[g][S-1];
+            // p0 = partner in class c0 (the fixed tile's runs are unused)
+            const int32_t p0 = fx ? u0 : wrap_m(2 * c0 + 1 - x, m);
+            const int32_t s0 = fx ? u0 : x;
+#pragma unroll
+            for (int32_t c = 0; c <= T; ++c) {
+              int32_t y0 = p0 + 2 * c, y1 = s0 + 2 * c;
+              y0 = y0 >= m ? y0 - m : y0;
+              y1 = y1 >= m ? y1 - m : y1;
+              cp_async4(dst + SM::R0 + c, row + y0);
+              cp_async4(dst + SM::R1 + c, row + y1);
+            }
+            cp_async4(dst + SM::CL, row + (S - 1));
+            // runU = E[g][u0 .. u0+2T+1] for the pair-0 light cone: local slots
+            // 0..Tp (first), nA..nA+Tp-1 (second), Lc-1 (S-1)
+            if (low && (j <= Tp || (j >= C.nA && j < C.nA + Tp) || fx)) {
+#pragma unroll
+              for (int32_t z = 0; z < SM::NU; ++z) {
+                int32_t y = u0 + z;
+                y = y >= m ? y - m : y;
+                cp_async4(dst + SM::RU + z, row + y);
+              }
+            }
+          }
+          cp_async_wait_all();
+        }
+        group_sync(1 + grp, GT);
+        if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
+        // ---- Tp classes on the extended range ----
+        if (have) {
+          for (int32_t t = 0; t < Tp; ++t) {
+            const int32_t lo = low ? 0 : C.a + t;
+            const int32_t hi = (C.b == K + 1) ? K + 1 : C.b - t;
+#pragma unroll
+            for (int q = 0; q < (X + 31) / 32; ++q) {
+              const int32_t kq = gt + GT * q;
+              const int32_t k = C.a + kq;
+              if (kq < X && k >= lo && k < hi) {
+                int32_t j1, j2;
+                C.local_slots(t, k, j1, j2);
+                const int4 A = s_st[j1], B = s_st[j2];
+                const int32_t e_bu = s_E[B.z];
+                const int32_t e_av = (k == 0) ? s_E[(A.x & 0xffff) * RS + SM::CL] : s_E[A.z];
+                const int32_t ia = A.x >> 16, ib = B.x >> 16;
+                if (A.y + B.y > e_bu + e_av) {
+                  if (k == 0) {   // B leaves S-1, A enters it
+                    const int32_t rb = (B.x & 0xffff) * RS + SM::RU + t + 2;
+                    s_st[j1] = make_int4((B.x & 0xffff) | (2 << 16), e_bu, rb, rb);
+                    s_st[j2] = make_int4((A.x & 0xffff) | (1 << 16), e_av,
+                                         (A.x & 0xffff) * RS + SM::RU + t + 1, 0);
+                  } else {
+                    s_st[j1] = make_int4(B.x, e_bu, B.w, B.z + ib);
+                    s_st[j2] = make_int4(A.x, e_av, A.w, A.z + ia);
+                  }
+                  if (k >= k0 && k < k1) ++mysw;
+                } else {
+                  s_st[j1] = make_int4(A.x, A.y, A.z + ia, A.w);
+                  s_st[j2] = make_int4(B.x, B.y, B.z + ib, B.w);
+                }
+              }
+              if (q + 1 >= (X + GT - 1) / GT) break;
+            }
+            group_sync(1 + grp, GT);
+          }
+        }
+        if (prof) { const unsigned long long t = gtimer(); t_st += t - tq; tq = t; }
+        // ---- write back the slots of the owned pairs (class c0 + Tp - 1) ----
+        if (have) {
+          for (int32_t kq = gt; kq < X; kq += GT) {
+            const int32_t k = C.a + kq;
+            if (k >= k0 && k < k1) {
+              int32_t j1, j2;
+              C.local_slots(Tp - 1, k, j1, j2);
+              const int32_t x1 = C.slot_of(j1, u0, S), x2 = C.slot_of(j2, u0, S);
+              const int4 A = s_st[j1], B = s_st[j2];
+              __stcg(rn + x1, s_g[A.x & 0xffff]);
+              __stcg(dn + x1, A.y);
+              __stcg(rn + x2, s_g[B.x & 0xffff]);
+              __stcg(dn + x2, B.y);
+            }
+          }
+        }
+        group_sync(1 + grp, GT);
+      }
+      // swaps of this phase -> the round counter
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) mysw += __shfl_xor_sync(0xffffffffu, mysw, o);
+      if ((threadIdx.x & 31) == 0 && mysw) atomicAdd(&s_cta_sw, mysw);
+      cur ^= 1;
+      bar_target += nblk;
+      __syncthreads();
+      if (threadIdx.x == 0 && s_cta_sw) {
+        atomicAdd(p.rsw + rounds % 3, (unsigned long long)s_cta_sw);
+        s_cta_sw = 0;
+      }
+      grid_barrier(p.bar, bar_target);
+      if (prof) { const unsigned long long t = gtimer(); t_bar += t - tq; tq = t; ++n_ph; }
+    }
+    // round end (Alg. 2 lines 10-11)
+    if (threadIdx.x == 0) s_rs = *((volatile unsigned long long*)(p.rsw + rounds % 3));
+    __syncthreads();
+    const int64_t rs = (int64_t)s_rs;
+    if (blockIdx.x == 0 && threadIdx.x == 0 && rounds < p.max_log) p.per_round[rounds] = rs;
+    rounds += 1;
+    total += rs;
+    __syncthreads();
+    if (rs == 0) break;
+    if (p.max_rounds > 0 && rounds >= p.max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
+    if (p.handoff && rs <= p.sparse_T) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) *p.handoff = 1;
+      break;
+    }
+  }
+  if (prof) {
+    p.per_round[192] = (int64_t)t_ld; p.per_round[193] = (int64_t)t_st;
+    p.per_round[194] = (int64_t)t_bar; p.per_round[195] = (int64_t)n_ph;
+  }
+  if (cur == 1) {   // the final state is in the scratch buffer: copy to perm
+    for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
+      p.rbuf[0][x] = __ldcg(p.rbuf[1] + x);
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    p.out->status = status;
+    p.out->rounds = rounds;
+    p.out->swaps = total;
+  }
+}
+
+static int32_t trap_env(const char* name, int32_t dflt) {
+  const char* s = std::getenv(name);
+  return (s && *s) ? (int32_t)std::atoi(s) : dflt;
+}
+
+int32_t ls_trap_min_S() { return 256; }
+
+template <int PPL, int T>
+static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
+  using SM = TrapSmem<PPL, T>;
+  constexpr int X = SM::X;
+  static_assert(X > 2 * T, "chunk must own at least one pair");
+  int dev = 0, nsm = 0, optin = 0;
+  PM_CUDA_TRY(cudaGetDevice(&dev));
+  PM_CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  PM_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  const Classes cl(hp.S);
+  const int32_t npairs = cl.npairs;
+  int32_t W = trap_env("PM_TRAP_W", X - 2 * T);
+  if (W < 1 || W > X - 2 * T) W = X - 2 * T;
+  hp.W = W;
+  hp.nchunks = (npairs + W - 1) / W;
+  // chunk groups of gsz warps (they stage a chunk together and split its
+  // pairs); cpc groups per CTA, enough CTAs to hold every chunk in one pass
+  int gsz = trap_env("PM_TRAP_GSZ", PPL >= 2 ? 2 : 1);
+  if (gsz < 1) gsz = 1;
+  if (gsz > 8) gsz = 8;
+  hp.gsz = gsz;
+  int max_cpc = (int)((size_t)optin / SM::bytes);
+  if (max_cpc > 8 / gsz) max_cpc = 8 / gsz;
+  if (max_cpc < 1) return PM_ERR_UNSUPPORTED;
+  int cpc = trap_env("PM_TRAP_CPC", (hp.nchunks + nsm - 1) / nsm);
+  if (cpc < 1) cpc = 1;
+  if (cpc > max_cpc) cpc = max_cpc;
+  const size_t smem = SM::bytes * cpc;
+  const int threads = 32 * gsz * cpc;
+  PM_CUDA_TRY(cudaFuncSetAttribute(k_ls_trap<PPL, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int occ = 0;
+  PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_ls_trap<PPL, T>, threads, smem));
+  if (occ < 1) return PM_ERR_UNSUPPORTED;
+  int grid = (hp.nchunks + cpc - 1) / cpc;
+  if (grid > nsm * occ) grid = nsm * occ;
+  void* args[] = {(void*)&hp};
+  PM_CUDA_TRY(cudaLaunchCooperativeKernel((const void*)k_ls_trap<PPL, T>, dim3(grid), dim3(threads), args, smem, st));
+  note_launch();
+  return PM_OK;
+}
+
+pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                     LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                     int32_t* handoff, int32_t sparse_T) {
+  if (S < ls_trap_min_S() || (S & 1)) return PM_ERR_UNSUPPORTED;
+  PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
+  // scratch: r1 [S], d0 [S], d1 [S], barrier counter, 3 round counters
+  const size_t n = (size_t)S;
+  char* scratch = nullptr;
+  const size_t bytes = sizeof(int32_t) * 3 * n + 64 + sizeof(unsigned long long) * 3;
+  PM_CUDA_TRY(pm::scratch_alloc(reinterpret_cast<void**>(&scratch), bytes, st));
+  unsigned long long* rsw = reinterpret_cast<unsigned long long*>(scratch);
+  unsigned int* bar = reinterpret_cast<unsigned int*>(scratch + 32);
+  int32_t* base = reinterpret_cast<int32_t*>(scratch + 64);
+  PM_CUDA_TRY(cudaMemsetAsync(scratch, 0, 64, st));
+  TrapParams hp = {};
+  hp.E = E; hp.ldE = ldE;
+  hp.rbuf[0] = perm; hp.rbuf[1] = base;
+  hp.dbuf[0] = base + n; hp.dbuf[1] = base + 2 * n;
+  hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
+  hp.sparse_T = sparse_T; hp.handoff = handoff;
+  hp.bar = bar; hp.rsw = rsw;
+  hp.out = dev_out; hp.per_round = dev_per_round;
+  hp.launches = device_launch_counter();
+  if (!hp.launches) return PM_ERR_CUDA;
+  hp.prof = trap_env("PM_TRAP_PROF", 0);
+  const int32_t variant = trap_env("PM_TRAP_V", 0);
+  pm_status_t s;
+  switch (variant) {
+    case 1: s = launch_trap<1, 8>(hp, st); break;
+    case 2: s = launch_trap<2, 8>(hp, st); break;
+    case 3: s = launch_trap<4, 16>(hp, st); break;
+    case 4: s = launch_trap<4, 8>(hp, st); break;
+    default: s = launch_trap<2, 16>(hp, st); break;
+  }
+  if (s != PM_OK) return s;
+  PM_CUDA_TRY(cudaFreeAsync(scratch, st));
+  return PM_OK;
+}
+
+int64_t trap_misses_read_and_reset() {
+  unsigned long long v = 0, z = 0;
+  if (cudaMemcpyFromSymbol(&v, g_trap_misses, sizeof(v)) != cudaSuccess) return -1;
+  if (cudaMemcpyToSymbol(g_trap_misses, &z, sizeof(z)) != cudaSuccess) return -1;
+  return (int64_t)v;
+}
+
+}  // namespace pm

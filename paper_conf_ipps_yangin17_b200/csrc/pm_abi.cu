@@ -95,7 +95,7 @@ struct DevBuf {
 bool valid_ls_args(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int32_t max_rounds,
                    int32_t method) {
   if (!d_E || !d_perm || S < 1 || ld_E < S || max_rounds < 0) return false;
-  return method >= PM_LS_AUTO && method <= PM_LS_WALK;
+  return method >= PM_LS_AUTO && method <= PM_LS_TRAP;
 }
 
 // Synchronous local search: scratch, launch, read back.
@@ -289,7 +289,7 @@ pm_status_t pm_photomosaic_async(const uint8_t* d_input, const uint8_t* d_target
                                  int32_t* d_E, int64_t ld_E, int32_t* d_perm, int32_t method, int64_t* d_result,
                                  pm_stream_t stream) {
   if (!d_input || !d_target || !d_E || !d_perm || !d_result || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
-  if (method < PM_LS_AUTO || method > PM_LS_WALK) return PM_ERR_INVALID;
+  if (method < PM_LS_AUTO || method > PM_LS_TRAP) return PM_ERR_INVALID;
   const int32_t g = N / M;
   const int32_t S = g * g;
   if (ld_E < S) return PM_ERR_INVALID;
@@ -375,6 +375,7 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
   return PM_OK;
 }
 
+int64_t pm_debug_trap_misses(void) { return trap_misses_read_and_reset(); }
 int64_t pm_launch_count(void) { return g_launches.load() + device_launch_total(); }
 
 }  // extern "C"

@@ -167,6 +167,13 @@ pm_status_t sparse_launch(SparseRun* run, cudaStream_t st);
 unsigned long long* device_launch_counter();
 int64_t device_launch_total();
 
+// Temporal-blocked whole-GPU search (k_trap.cu).
+int32_t ls_trap_min_S();
+pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
+                     LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
+                     int32_t* handoff, int32_t sparse_T);
+int64_t trap_misses_read_and_reset();
+
 // Exact min-weight perfect matching by eps-scaling auction (k_assign.cu).
 // h_stats (nullable): {bidding rounds, phases}.  Synchronises st.
 pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* perm, int64_t* price_out,

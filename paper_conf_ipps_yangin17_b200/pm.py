@@ -20,7 +20,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libpm.so")
 
 PM_OK, PM_ERR_INVALID, PM_ERR_CUDA, PM_ERR_NOT_CONVERGED, PM_ERR_UNSUPPORTED, PM_ERR_NOT_PERMUTATION = range(6)
-METHODS = {"auto": 0, "class": 1, "cta": 2, "window": 3, "pairwin": 4, "walk": 5}
+METHODS = {"auto": 0, "class": 1, "cta": 2, "window": 3, "pairwin": 4, "walk": 5, "trap": 6}
 
 _lib = None
 _P = ctypes.c_void_p
@@ -49,6 +49,7 @@ _SIGS = [
     ("pm_render", ctypes.c_int, [_P, _I32, _I32, _I32, _P, _P, _P]),
     ("pm_optimal_assignment", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P, _P, _P]),
     ("pm_launch_count", _I64, []),
+    ("pm_debug_trap_misses", _I64, []),
 ]
 
 

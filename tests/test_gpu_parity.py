@@ -132,7 +132,8 @@ def test_error_matrix_config5_row_chunks_sampled():
 
 # ------------------------------------------------------------------ Alg. 2 --
 def _supported(method, S):
-    return not (method == "pairwin" and not (40 <= S <= 2048)) and not (method == "window" and S > 2048)
+    return (not (method == "pairwin" and not (40 <= S <= 2048)) and not (method == "window" and S > 2048)
+            and not (method == "trap" and (S < 256 or S % 2)))
 
 
 def _check_ls(E_np, method, perm0=None, max_rounds=0):
@@ -150,39 +151,39 @@ def _check_ls(E_np, method, perm0=None, max_rounds=0):
     return ref
 
 
-@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "shuffle", "transposition", "identical"])
 def test_local_search_parity_config1(method, fam):
     _check_ls(oracle_E(fam, 128, 8), method)
 
 
-@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
 def test_local_search_parity_config2(method, fam):
     _check_ls(oracle_E(fam, 512, 16), method)
 
 
-@pytest.mark.parametrize("method", ["auto", "walk", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "trap", "walk", "cta", "class"])
 def test_local_search_parity_config3(method):
     ref = _check_ls(oracle_E("smooth", 1024, 16), method)
     assert ref[1] >= 3
 
 
-@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
 @pytest.mark.parametrize("N,M,C", [(90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (30, 10, 3), (64, 64, 1)])
 def test_local_search_parity_ragged_and_odd(method, N, M, C):
     # S = 81, 49, 9 are odd (the fixed point idles, reading R9); S = 1 trivial
     _check_ls(oracle_E("smooth", N, M, C), method)
 
 
-@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
 def test_local_search_resume_from_any_bijection(method):
     E = oracle_E("noise", 128, 8)
     rng = np.random.default_rng(3)
     _check_ls(E, method, perm0=rng.permutation(256).astype(np.int32))
 
 
-@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
 def test_local_search_max_rounds_then_resume(method):
     E_np = oracle_E("smooth", 512, 16)
     ref = _check_ls(E_np, method, max_rounds=2)
@@ -190,7 +191,7 @@ def test_local_search_max_rounds_then_resume(method):
     _check_ls(E_np, method, perm0=ref[0])
 
 
-@pytest.mark.parametrize("method", ["walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
 def test_local_search_rejects_non_permutation(method):
     E = dev(oracle_E("smooth", 128, 8))
     bad = torch.arange(256, dtype=torch.int32, device=DEV)
@@ -270,7 +271,7 @@ def test_cost_int64():
 
 
 # -------------------------------------------------------------- pipeline ----
-@pytest.mark.parametrize("method", ["auto", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "trap", "pairwin", "window", "cta", "class"])
 def test_photomosaic_pipeline_config2(method):
     I, T = pair("smooth", 512, 16)
     E_np = oracle_E("smooth", 512, 16)
@@ -490,3 +491,29 @@ def test_walk_mailbox_overflow_falls_back_exactly():
     E_np = oracle.error_matrix(I, Tt, M)
     ref = _check_ls(E_np, "walk")
     assert ref[3][0] >= 63
+
+
+# ---- PM_LS_TRAP: every round on the temporal-blocked kernel (sparse hand-over
+# off), every compiled (pairs-per-lane, T) variant, chunk widths that do not
+# divide S/2, and no E lookup outside the staged runs.
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("N,M,fam,W", [(128, 8, "smooth", 0), (512, 16, "smooth", 0), (512, 16, "ties", 7),
+                                       (240, 8, "noise", 0), (336, 8, "smooth", 5), (128, 8, "transposition", 3)])
+def test_trap_every_round(variant, N, M, fam, W, monkeypatch):
+    monkeypatch.setenv("PM_TRAP_V", str(variant))
+    monkeypatch.setenv("PM_LS_SPARSE", "0")
+    monkeypatch.setenv("PM_TRAP_W", str(W))
+    pm.lib().pm_debug_trap_misses()
+    _check_ls(oracle_E(fam, N, M), "trap")
+    assert pm.lib().pm_debug_trap_misses() == 0
+
+
+@pytest.mark.parametrize("cpc,gsz,variant", [(1, 1, 0), (2, 2, 0), (3, 1, 1), (1, 4, 3), (2, 4, 4), (1, 8, 2)])
+def test_trap_warps_per_cta(cpc, gsz, variant, monkeypatch):
+    monkeypatch.setenv("PM_TRAP_CPC", str(cpc))
+    monkeypatch.setenv("PM_TRAP_GSZ", str(gsz))
+    monkeypatch.setenv("PM_TRAP_V", str(variant))
+    monkeypatch.setenv("PM_LS_SPARSE", "0")
+    pm.lib().pm_debug_trap_misses()
+    _check_ls(oracle_E("noise", 1024, 16), "trap")
+    assert pm.lib().pm_debug_trap_misses() == 0
