@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--family", default="smooth")
-    ap.add_argument("--method", default="auto", choices=["auto", "class", "cta", "window", "pairwin"])
+    ap.add_argument("--method", default="auto", choices=["auto", "trap", "class", "cta", "window", "pairwin", "walk"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="budget of the cpu_baseline sample")
     ap.add_argument("--e2e-steps", type=int, default=10)
@@ -269,8 +269,10 @@ def bench_ours(args, rank, world, local_rank):
     ls_gbs = ls_bytes / (mean_ls * 1e-3) / 1e9
     e_tops = S * S * P / (mean_e * 1e-3) / 1e12
     used = pm.ls_auto_method(S) if args.method == "auto" else args.method
-    ls_kernel = {"window": "k_ls_window (+ k_permute_cols)", "cta": "k_ls_cta",
-                 "class": "k_ls_class x (S-1) per round (CUDA graph)"}[used]
+    ls_kernel = {"trap": "k_ls_trap (temporal-blocked class replay, dense rounds) + sparse rounds",
+                 "window": "k_ls_window (+ k_permute_cols) + sparse rounds", "cta": "k_ls_cta",
+                 "class": "k_ls_class x (S-1) per round (CUDA graph) + sparse rounds",
+                 "pairwin": "k_pw_* rounds", "walk": "k_sp_scan + k_sp_walk rounds"}[used]
     traffic = {}
     try:
         traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
@@ -283,7 +285,7 @@ def bench_ours(args, rank, world, local_rank):
 
     roof_ls = {"kernel": f"{ls_kernel}: Alg. 2, all rounds", "bound": "hbm", "achieved": ls_gbs,
                "peak": hbm_peak, "unit": "GB/s", "frac": ls_gbs / hbm_peak,
-               "traffic": _traffic("k_ls_" + used) if used in ("window", "cta") else None,
+               "traffic": _traffic("k_ls_" + used) if used in ("trap", "window", "cta") else None,
                "peak_source": hbm_src, "algorithmic_bytes": ls_bytes,
                "note": "latency-bound dependency chain of S-1 class steps per round; bytes = rounds*S(S-1)/2*8"}
     roof_e = {"kernel": "k_sad (Eq. 1; Step 1 fused into its loader at S <= 4096)", "bound": "alu",

@@ -251,11 +251,6 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
  * device counter back and synchronises with the devices it has used. */
 int64_t pm_launch_count(void);
 
-/* Test hook: E lookups PM_LS_TRAP had to serve from global memory because
- * they fell outside the staged runs (expected 0; the result is exact either
- * way) since the last call.  Synchronises the current device; -1 on error. */
-int64_t pm_debug_trap_misses(void);
-
 #ifdef __cplusplus
 }
 #endif

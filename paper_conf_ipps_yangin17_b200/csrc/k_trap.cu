@@ -1,5 +1,5 @@
-// k_trap.cu -- Algorithm 2 on the whole GPU by temporal blocking
-// of the colour-class sequence (method PM_LS_TRAP).
+// k_trap.cu -- Algorithm 2 on many SMs by temporal blocking of
+// the colour-class sequence (method PM_LS_TRAP).
 //
 // Structure used.  Class c pairs slot u0+k with u0-k (mod m), k = 1..K, and
 // u0 with S-1 (k = 0), where u0 = c + (m+1)/2 and K = S/2 - 1 (Theorem 1,
@@ -11,47 +11,55 @@
 // class index.  Alg. 2's exact result for the pairs [k0, k1) after T more
 // classes is a function of the state of pairs [k0-T, k1+T) alone.
 //
-// Kernel.  One persistent cooperative grid.  A phase covers T consecutive
-// classes of a round.  The pairs are cut into chunks of W owned pairs; a warp
-// takes a chunk, copies the state (r, d) of the slots of its extended range
-// [k0-T, k1+T) into shared memory, replays the T classes on it (the valid
-// range shrinks by one pair per side and class, "overlapped tiling") and
-// writes back the slots of its owned pairs.  Phases are separated by a grid
-// barrier, state ping-pongs between two global buffers.  Each pair test is
-// line 5 with two entries carried in d (as every other method here):
-// d[u] + d[v] > E[r[v]][u] + E[r[u]][v], strict (R6).
+// Kernel.  A phase covers T consecutive classes of a round.  The pairs are cut
+// into chunks of W owned pairs; a group of warps takes a chunk, copies the
+// state (r, d) of the slots of its extended range [k0-T, k1+T) into shared
+// memory, replays the T classes on it (the valid range shrinks by one pair per
+// side and class: overlapped tiling) and publishes the slots of its owned
+// pairs.  Two modes:
+//   grid    -- persistent cooperative grid; state ping-pongs between two
+//              global buffers, one grid barrier per phase (any S).
+//   cluster -- one thread-block cluster (<= 16 CTAs) holds every chunk; each
+//              CTA keeps replicas of r and d, published slots go to the
+//              replicas of the CTAs of the neighbouring chunks by DSMEM
+//              stores, one cluster barrier per phase (small S).
+// Each pair test is line 5 with two entries carried in d (as every method
+// here): d[u] + d[v] > E[r[v]][u] + E[r[u]][v], strict (R6).
 //
-// E entries a chunk can need.  A tile starting at slot s0 whose class-c0
-// partner is p0 only ever sits at, or is tested against, slots s0 + 2j and
-// p0 + 2j (j < T) while it stays away from pair 0: the partner of slot x in
-// class c is 2c+1-x.  Through pair 0 (chunks with k0 <= T) it can also meet
-// u0 .. u0+2T and S-1.  So each tile of the chunk gets two stride-2 runs of T
-// entries of its E row, E[t][S-1], and for the first chunk(s) the contiguous
-// run E[t][u0 .. u0+2T]: O(T) entries per tile instead of the O(W+2T) of a
-// full sub-block.  A lookup outside the runs (never expected) falls back to a
-// global load and is counted (pm_debug_trap_misses), so the result is exact
-// regardless.
+// E entries a chunk needs.  The partner of slot y in class c is 2c+1-y
+// (mod m), so a tile that stays at y meets partners advancing by 2 per class,
+// and after a swap its new partner is its old slot + 2.  A tile starting at
+// slot s0 with class-c0 partner p0 is thus only ever tested against slots
+// p0 + 2j and s0 + 2j (j <= T) -- two stride-2 runs of its E row -- unless it
+// passes through pair 0 (slot S-1 meets u0, u0+1, ...), which only tiles
+// within T pairs of pair 0 can reach: for them the contiguous run
+// E[t][u0 .. u0+2T+1] is staged too, and E[t][S-1] for every tile.  Each slot
+// state carries indices of the staged entries of its tile's current partner
+// (pp) and of slot + 2 (po): no swap -> pp += inc; swap -> (pp, po) <- (po,
+// pp + inc) -- inc = 1 in a compact stride-2 run, 2 in the contiguous run.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
+#include <cstdio>
 #include <cstdlib>
 
 #include "pm_internal.cuh"
 
-namespace pm {
+namespace cg = cooperative_groups;
 
-__device__ unsigned long long g_trap_misses;
+namespace pm {
 
 struct TrapParams {
   const int32_t* E;
   int64_t ldE;
-  int32_t* rbuf[2];            // rbuf[0] = the caller's perm
+  int32_t* rbuf[2];            // rbuf[0] = the caller's perm (grid mode: ping-pong)
   int32_t* dbuf[2];
   int32_t S, max_rounds, max_log, sparse_T;
   int32_t W, nchunks;
-  int32_t gsz;                 // warps per chunk group
-  int32_t prof;                // PM_TRAP_PROF: block 0 thread 0 phase timers -> per_round[192..195]
+  int32_t gsz;                 // warps per chunk group (= PPL)
+  int32_t prof;                // PM_TRAP_PROF: CTA 0 thread 0 phase timers -> per_round[192..195]
   unsigned int* bar;           // grid barrier counter (zeroed before launch)
-  unsigned long long* rsw;     // [3] swaps per round, rotating
+  unsigned long long* rsw;     // [3] swaps per round, rotating (grid mode)
   LsResult* out;
   int64_t* per_round;
   int32_t* handoff;
@@ -63,13 +71,13 @@ struct TrapSmem {
   static constexpr int X = 32 * PPL;        // pairs of an extended range
   static constexpr int L = 2 * X;           // slots (= tiles) of an extended range
   // staged row of local tile i: run0 [R0, R0+T+1) = E[g][p0 + 2j], run1
-  // [R1, R1+T+1) = E[g][s0 + 2j], E[g][S-1] at CL, runU [RU, RU+2T+2) =
-  // E[g][u0 + z] (pair-0 light cone only); odd stride (banks)
-  static constexpr int R0 = 0, R1 = T + 1, CL = 2 * T + 2, RU = 2 * T + 3;
-  static constexpr int NE = 2 * T + 3;      // entries staged for every tile
-  static constexpr int NU = 2 * T + 2;      // runU entries
-  static constexpr int RS = 4 * T + 5;
-  static constexpr int ints = L * (4 + 1 + RS);   // int4 state + g + rows
+  // [R1, R1+T+1) = E[g][s0 + 2j], E[g][S-1] at CL; odd stride (banks)
+  static constexpr int R0 = 0, R1 = T + 1, CL = 2 * T + 2;
+  static constexpr int RS = 2 * T + 3;
+  static constexpr int NC = 2 * T + 2;      // pair-0 light-cone tiles (at most)
+  static constexpr int NU = 2 * T + 3;      // their runU = E[g][u0 + z], z <= 2T+1 (odd stride)
+  static constexpr int UOFF = L * RS;       // cone rows follow the rows (one index space)
+  static constexpr int ints = (L * (4 + 1 + RS) + NC * NU + 3) / 4 * 4;   // int4 state + g + rows + cone rows
   static constexpr size_t bytes = sizeof(int32_t) * (size_t)ints;
 };
 
@@ -115,7 +123,7 @@ __device__ __forceinline__ void grid_barrier(unsigned int* bar, unsigned int tar
 // j = nA + nB -> S - 1 (only when a == 0).  Pair k at step t (class c0 + t)
 // has slots u0 + t + k and u0 + t - k (or S - 1 for k = 0).
 struct TrapChunk {
-  int32_t a, b, a2, nA, nB, Lc, K, m;
+  int32_t a, b, a2, nA, nB, Lc, K, m, Tp;
   __device__ __forceinline__ void local_slots(int32_t t, int32_t k, int32_t& j1, int32_t& j2) const {
     const int32_t o1 = t + k;
     j1 = (o1 <= K) ? o1 - a : nA + (m - o1 - a2);
@@ -127,36 +135,123 @@ struct TrapChunk {
     if (j < nA + nB) return wrap_m(u0 - (a2 + j - nA), m);
     return S - 1;
   }
+  // index of local tile i in the pair-0 light cone (low chunks), -1 if outside:
+  // local slots 0..Tp (first), nA..nA+Tp-1 (second), Lc-1 (S-1)
+  __device__ __forceinline__ int32_t cone(int32_t i) const {
+    if (a != 0) return -1;
+    if (i <= Tp) return i;
+    if (i >= nA && i < nA + Tp) return Tp + 1 + (i - nA);
+    if (i == Lc - 1) return 2 * Tp + 1;
+    return -1;
+  }
 };
 
-// State of a slot: {tile | inc << 16, d, pp, po}: pp indexes the staged
-// E[tile][partner of the slot in the current class], po the staged
-// E[tile][slot + 2].  The partner of slot y in class c is 2c+1-y (mod m), so
-// while a tile stays its partner advances by 2 (pp += inc: consecutive
-// entries of a stride-2 run, inc = 1, or of runU, inc = 2) and after a swap
-// its new partner is its old slot + 2 (pp <- po, po <- pp + inc).  The slot
-// S-1 (pair 0) walks u0, u0+1, ... through runU with inc = 1.
-template <int PPL, int T>
+// One chunk of one phase: stage (state via `src`, E rows from global), replay
+// Tp classes.  Returns the swaps of the owned pairs.
+template <int PPL, int T, typename Src>
+__device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_t k1, int32_t c0, int32_t u0,
+                                          const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
+                                          int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
+                                          unsigned long long* tprof) {
+  using SM = TrapSmem<PPL, T>;
+  constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
+  const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
+  const bool low = (C.a == 0);
+  int32_t* s_U = s_E + SM::UOFF;
+  // ---- one thread per local slot j (= local tile j): its state, then its
+  // tile's E row pieces, every copy independent of the others ----
+  for (int32_t j = gt; j < Lc; j += GT) {
+    const int32_t x = C.slot_of(j, u0, S);
+    int32_t g, d;
+    src(x, g, d);
+    s_g[j] = g;
+    const bool fx = (x == S - 1);
+    const int32_t ci = C.cone(j);
+    s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU, 0)
+                 : make_int4(j | (1 << 16), d, j * RS + SM::R0, j * RS + SM::R1 + 1);
+    const int32_t* row = E + (int64_t)g * ld;
+    int32_t* dst = s_E + j * RS;
+    // run0: E[g][p0 + 2c], run1: E[g][x + 2c] (c <= T), E[g][S-1];
+    // p0 = partner in class c0 (the fixed tile's runs are unused)
+    const int32_t p0 = fx ? u0 : wrap_m(2 * c0 + 1 - x, m);
+    const int32_t s0 = fx ? u0 : x;
+#pragma unroll
+    for (int32_t c = 0; c <= T; ++c) {
+      int32_t y0 = p0 + 2 * c, y1 = s0 + 2 * c;
+      y0 = y0 >= m ? y0 - m : y0;
+      y1 = y1 >= m ? y1 - m : y1;
+      cp_async4(dst + SM::R0 + c, row + y0);
+      cp_async4(dst + SM::R1 + c, row + y1);
+    }
+    cp_async4(dst + SM::CL, row + (S - 1));
+    if (ci >= 0) {
+      int32_t* du = s_U + ci * SM::NU;
+#pragma unroll
+      for (int32_t z = 0; z < 2 * T + 2; ++z) {
+        int32_t y = u0 + z;
+        y = y >= m ? y - m : y;
+        cp_async4(du + z, row + y);
+      }
+    }
+  }
+  cp_async_wait_all();
+  group_sync(bar_id, GT);
+  unsigned long long t0 = tprof ? gtimer() : 0;
+  // ---- Tp classes on the extended range: thread gt takes pair a + gt ----
+  int mysw = 0;
+  const int32_t k = C.a + gt;
+  const bool own = (k >= k0 && k < k1);
+  for (int32_t t = 0; t < Tp; ++t) {
+    const int32_t lo = low ? 0 : C.a + t;
+    const int32_t hi = (C.b == K + 1) ? K + 1 : C.b - t;
+    if (k >= lo && k < hi) {
+      int32_t j1, j2;
+      C.local_slots(t, k, j1, j2);
+      const int4 A = s_st[j1], B = s_st[j2];
+      const int32_t e_bu = s_E[B.z];
+      const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z];
+      const int32_t ia = A.x >> 16, ib = B.x >> 16;
+      const bool sw = A.y + B.y > e_bu + e_av;
+      int4 nA = sw ? make_int4(B.x, e_bu, B.w, B.z + ib) : make_int4(A.x, A.y, A.z + ia, A.w);
+      int4 nB = sw ? make_int4(A.x, e_av, A.w, A.z + ia) : make_int4(B.x, B.y, B.z + ib, B.w);
+      if (k == 0 && sw) {   // B leaves S-1 for slot u0+t (next partner u0+t+2), A enters S-1
+        const int32_t rb = SM::UOFF + C.cone(B.x & 0xffff) * SM::NU + t + 2;
+        nA = make_int4((B.x & 0xffff) | (2 << 16), e_bu, rb, rb);
+        nB = make_int4((A.x & 0xffff) | (1 << 16), e_av, SM::UOFF + C.cone(A.x & 0xffff) * SM::NU + t + 1, 0);
+      }
+      s_st[j1] = nA;
+      s_st[j2] = nB;
+      mysw += (sw && own) ? 1 : 0;
+    }
+    group_sync(bar_id, GT);
+  }
+  if (tprof) *tprof += gtimer() - t0;
+  return mysw;
+}
+
+template <int PPL, int T, bool CLU>
 __global__ void __launch_bounds__(256, 1)
 k_ls_trap(const TrapParams p) {
   using SM = TrapSmem<PPL, T>;
-  constexpr int L = SM::L, RS = SM::RS, X = SM::X;
+  constexpr int L = SM::L, X = SM::X;
   extern __shared__ __align__(16) int32_t sm[];
-  const int gsz = p.gsz;                       // warps per chunk group
-  const int cpc = (blockDim.x >> 5) / gsz;     // chunk groups per CTA
-  const int grp = (threadIdx.x >> 5) / gsz;
-  const int GT = 32 * gsz;
+  constexpr int GT = X;                        // threads per chunk group (PPL warps)
+  const int cpc = blockDim.x / GT;             // chunk groups per CTA
+  const int grp = threadIdx.x / GT;
   const int gt = threadIdx.x - grp * GT;
   int32_t* ws = sm + (size_t)grp * SM::ints;
   int4* s_st = reinterpret_cast<int4*>(ws);
   int32_t* s_g = ws + 4 * L;
   int32_t* s_E = s_g + L;
+  const int32_t S = p.S;
+  // cluster mode: replicas of r and d, ping-pong [2][S] each
+  int32_t* rep_r = sm + (size_t)cpc * SM::ints;
+  int32_t* rep_d = rep_r + 2 * S;
   __shared__ int32_t s_cta_sw;
-  __shared__ unsigned long long s_rs;
+  __shared__ unsigned long long s_rs, s_rsw[3];
 
   const int32_t* __restrict__ E = p.E;
   const int64_t ld = p.ldE;
-  const int32_t S = p.S;
   const Classes cl(S);
   const int32_t m = cl.m, H = cl.half, K = cl.npairs - 1, ncls = cl.ncls;
   const int32_t W = p.W;
@@ -168,12 +263,21 @@ k_ls_trap(const TrapParams p) {
   if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.launches, 1ull);
   if (p.out->status != PM_OK) return;   // grid-uniform (written before launch)
 
-  if (threadIdx.x == 0) s_cta_sw = 0;
+  if (threadIdx.x == 0) { s_cta_sw = 0; s_rsw[0] = s_rsw[1] = s_rsw[2] = 0ull; }
   // d[x] = E[r[x]][x] (the maintained diagonal)
-  for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
-    __stcg(p.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(p.rbuf[0] + x) * ld + x));
-  bar_target += nblk;
-  grid_barrier(p.bar, bar_target);
+  if (CLU) {
+    for (int32_t x = threadIdx.x; x < S; x += blockDim.x) {
+      const int32_t g = __ldcg(p.rbuf[0] + x);
+      rep_r[x] = g;
+      rep_d[x] = __ldg(E + (int64_t)g * ld + x);
+    }
+    cg::this_cluster().sync();
+  } else {
+    for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
+      __stcg(p.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(p.rbuf[0] + x) * ld + x));
+    bar_target += nblk;
+    grid_barrier(p.bar, bar_target);
+  }
 
   int cur = 0;
   int32_t rounds = 0;
@@ -183,14 +287,13 @@ k_ls_trap(const TrapParams p) {
   unsigned long long t_ld = 0, t_st = 0, t_bar = 0, n_ph = 0, tq = prof ? gtimer() : 0;
   const int npass = (p.nchunks + ngrp_tot - 1) / ngrp_tot;
   for (;;) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      if (CLU) s_rsw[(rounds + 1) % 3] = 0ull;
+      else p.rsw[(rounds + 1) % 3] = 0ull;
+    }
     for (int32_t c0 = 0; c0 < ncls; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
       const int32_t u0 = wrap_m(c0 + H, m);
-      const int32_t* __restrict__ rc = cur ? p.rbuf[1] : p.rbuf[0];
-      const int32_t* __restrict__ dc = cur ? p.dbuf[1] : p.dbuf[0];
-      int32_t* rn = cur ? p.rbuf[0] : p.rbuf[1];
-      int32_t* dn = cur ? p.dbuf[0] : p.dbuf[1];
       int mysw = 0;
       for (int pass = 0; pass < npass; ++pass) {
         const int32_t ch = gid + pass * ngrp_tot;
@@ -200,91 +303,24 @@ k_ls_trap(const TrapParams p) {
         C.a = max(k0 - Tp, 0); C.b = min(k1 + Tp, K + 1);
         C.a2 = max(C.a, 1);
         C.nA = C.b - C.a; C.nB = C.b - C.a2;
-        const bool low = (C.a == 0);
-        C.Lc = C.nA + C.nB + (low ? 1 : 0);
-        C.K = K; C.m = m;
-        const int32_t Lc = C.Lc;
+        C.Lc = C.nA + C.nB + (C.a == 0 ? 1 : 0);
+        C.K = K; C.m = m; C.Tp = Tp;
         if (have) {
-          // ---- one thread per local slot j (= local tile j): its state, then
-          // its tile's E row pieces, every copy independent of the others ----
-          for (int32_t j = gt; j < Lc; j += GT) {
-            const int32_t x = C.slot_of(j, u0, S);
-            const int32_t g = __ldcg(rc + x);
-            const int32_t d = __ldcg(dc + x);
-            s_g[j] = g;
-            const bool fx = (x == S - 1);
-            s_st[j] = fx ? make_int4(j | (1 << 16), d, j * RS + SM::RU, 0)
-                         : make_int4(j | (1 << 16), d, j * RS + SM::R0, j * RS + SM::R1 + 1);
-            const int32_t* row = E + (int64_t)g * ld;
-            int32_t* dst = s_E + j * RS;
-            // run0: E[g][p0 + 2c], run1: E[g][x + 2c] (c <= T), E[g][S-1];
-            // p0 = partner in class c0 (the fixed tile's runs are unused)
-            const int32_t p0 = fx ? u0 : wrap_m(2 * c0 + 1 - x, m);
-            const int32_t s0 = fx ? u0 : x;
-#pragma unroll
-            for (int32_t c = 0; c <= T; ++c) {
-              int32_t y0 = p0 + 2 * c, y1 = s0 + 2 * c;
-              y0 = y0 >= m ? y0 - m : y0;
-              y1 = y1 >= m ? y1 - m : y1;
-              cp_async4(dst + SM::R0 + c, row + y0);
-              cp_async4(dst + SM::R1 + c, row + y1);
-            }
-            cp_async4(dst + SM::CL, row + (S - 1));
-            // runU = E[g][u0 .. u0+2T+1] for the pair-0 light cone: local slots
-            // 0..Tp (first), nA..nA+Tp-1 (second), Lc-1 (S-1)
-            if (low && (j <= Tp || (j >= C.nA && j < C.nA + Tp) || fx)) {
-#pragma unroll
-              for (int32_t z = 0; z < SM::NU; ++z) {
-                int32_t y = u0 + z;
-                y = y >= m ? y - m : y;
-                cp_async4(dst + SM::RU + z, row + y);
-              }
-            }
+          if (CLU) {
+            const int32_t* rr = rep_r + cur * S;
+            const int32_t* rd = rep_d + cur * S;
+            mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
+                                       [&](int32_t x, int32_t& g, int32_t& d) { g = rr[x]; d = rd[x]; },
+                                       s_st, s_g, s_E, gt, 1 + grp, prof ? &t_st : nullptr);
+          } else {
+            const int32_t* __restrict__ rc = cur ? p.rbuf[1] : p.rbuf[0];
+            const int32_t* __restrict__ dc = cur ? p.dbuf[1] : p.dbuf[0];
+            mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
+                                       [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
+                                       s_st, s_g, s_E, gt, 1 + grp, prof ? &t_st : nullptr);
           }
-          cp_async_wait_all();
-        }
-        group_sync(1 + grp, GT);
-        if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
-        // ---- Tp classes on the extended range ----
-        if (have) {
-          for (int32_t t = 0; t < Tp; ++t) {
-            const int32_t lo = low ? 0 : C.a + t;
-            const int32_t hi = (C.b == K + 1) ? K + 1 : C.b - t;
-#pragma unroll
-            for (int q = 0; q < (X + 31) / 32; ++q) {
-              const int32_t kq = gt + GT * q;
-              const int32_t k = C.a + kq;
-              if (kq < X && k >= lo && k < hi) {
-                int32_t j1, j2;
-                C.local_slots(t, k, j1, j2);
-                const int4 A = s_st[j1], B = s_st[j2];
-                const int32_t e_bu = s_E[B.z];
-                const int32_t e_av = (k == 0) ? s_E[(A.x & 0xffff) * RS + SM::CL] : s_E[A.z];
-                const int32_t ia = A.x >> 16, ib = B.x >> 16;
-                if (A.y + B.y > e_bu + e_av) {
-                  if (k == 0) {   // B leaves S-1, A enters it
-                    const int32_t rb = (B.x & 0xffff) * RS + SM::RU + t + 2;
-                    s_st[j1] = make_int4((B.x & 0xffff) | (2 << 16), e_bu, rb, rb);
-                    s_st[j2] = make_int4((A.x & 0xffff) | (1 << 16), e_av,
-                                         (A.x & 0xffff) * RS + SM::RU + t + 1, 0);
-                  } else {
-                    s_st[j1] = make_int4(B.x, e_bu, B.w, B.z + ib);
-                    s_st[j2] = make_int4(A.x, e_av, A.w, A.z + ia);
-                  }
-                  if (k >= k0 && k < k1) ++mysw;
-                } else {
-                  s_st[j1] = make_int4(A.x, A.y, A.z + ia, A.w);
-                  s_st[j2] = make_int4(B.x, B.y, B.z + ib, B.w);
-                }
-              }
-              if (q + 1 >= (X + GT - 1) / GT) break;
-            }
-            group_sync(1 + grp, GT);
-          }
-        }
-        if (prof) { const unsigned long long t = gtimer(); t_st += t - tq; tq = t; }
-        // ---- write back the slots of the owned pairs (class c0 + Tp - 1) ----
-        if (have) {
+          if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
+          // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
           for (int32_t kq = gt; kq < X; kq += GT) {
             const int32_t k = C.a + kq;
             if (k >= k0 && k < k1) {
@@ -292,10 +328,30 @@ k_ls_trap(const TrapParams p) {
               C.local_slots(Tp - 1, k, j1, j2);
               const int32_t x1 = C.slot_of(j1, u0, S), x2 = C.slot_of(j2, u0, S);
               const int4 A = s_st[j1], B = s_st[j2];
-              __stcg(rn + x1, s_g[A.x & 0xffff]);
-              __stcg(dn + x1, A.y);
-              __stcg(rn + x2, s_g[B.x & 0xffff]);
-              __stcg(dn + x2, B.y);
+              const int32_t g1 = s_g[A.x & 0xffff], g2 = s_g[B.x & 0xffff];
+              if (CLU) {
+                // to the replicas of the CTAs of chunks ch-1, ch, ch+1 (every slot of
+                // a chunk's next extended range is published by one of them: W > T)
+                cg::cluster_group cgc = cg::this_cluster();
+                const int nx = cur ^ 1;
+                int lastb = -1;
+                for (int dch = -1; dch <= 1; ++dch) {
+                  const int32_t c2 = ch + dch;
+                  if (c2 < 0 || c2 >= p.nchunks) continue;
+                  const int blk = c2 / cpc;
+                  if (blk == lastb) continue;
+                  lastb = blk;
+                  int32_t* rr = cgc.map_shared_rank(rep_r, blk) + nx * S;
+                  int32_t* rd = cgc.map_shared_rank(rep_d, blk) + nx * S;
+                  rr[x1] = g1; rd[x1] = A.y;
+                  rr[x2] = g2; rd[x2] = B.y;
+                }
+              } else {
+                int32_t* rn = cur ? p.rbuf[0] : p.rbuf[1];
+                int32_t* dn = cur ? p.dbuf[0] : p.dbuf[1];
+                __stcg(rn + x1, g1); __stcg(dn + x1, A.y);
+                __stcg(rn + x2, g2); __stcg(dn + x2, B.y);
+              }
             }
           }
         }
@@ -306,23 +362,32 @@ k_ls_trap(const TrapParams p) {
       for (int o = 16; o > 0; o >>= 1) mysw += __shfl_xor_sync(0xffffffffu, mysw, o);
       if ((threadIdx.x & 31) == 0 && mysw) atomicAdd(&s_cta_sw, mysw);
       cur ^= 1;
-      bar_target += nblk;
       __syncthreads();
       if (threadIdx.x == 0 && s_cta_sw) {
-        atomicAdd(p.rsw + rounds % 3, (unsigned long long)s_cta_sw);
+        if (CLU) atomicAdd(cg::this_cluster().map_shared_rank(&s_rsw[rounds % 3], 0), (unsigned long long)s_cta_sw);
+        else atomicAdd(p.rsw + rounds % 3, (unsigned long long)s_cta_sw);
         s_cta_sw = 0;
       }
-      grid_barrier(p.bar, bar_target);
+      if (CLU) {
+        cg::this_cluster().sync();
+      } else {
+        bar_target += nblk;
+        grid_barrier(p.bar, bar_target);
+      }
       if (prof) { const unsigned long long t = gtimer(); t_bar += t - tq; tq = t; ++n_ph; }
     }
     // round end (Alg. 2 lines 10-11)
-    if (threadIdx.x == 0) s_rs = *((volatile unsigned long long*)(p.rsw + rounds % 3));
+    if (threadIdx.x == 0) {
+      if (CLU) s_rs = *cg::this_cluster().map_shared_rank(&s_rsw[rounds % 3], 0);
+      else s_rs = *((volatile unsigned long long*)(p.rsw + rounds % 3));
+    }
     __syncthreads();
     const int64_t rs = (int64_t)s_rs;
     if (blockIdx.x == 0 && threadIdx.x == 0 && rounds < p.max_log) p.per_round[rounds] = rs;
     rounds += 1;
     total += rs;
-    __syncthreads();
+    if (CLU) cg::this_cluster().sync();   // CTA 0 resets the next counter only after every read
+    else __syncthreads();
     if (rs == 0) break;
     if (p.max_rounds > 0 && rounds >= p.max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
     if (p.handoff && rs <= p.sparse_T) {
@@ -331,10 +396,25 @@ k_ls_trap(const TrapParams p) {
     }
   }
   if (prof) {
-    p.per_round[192] = (int64_t)t_ld; p.per_round[193] = (int64_t)t_st;
+    p.per_round[192] = (int64_t)(t_ld - t_st); p.per_round[193] = (int64_t)t_st;
     p.per_round[194] = (int64_t)t_bar; p.per_round[195] = (int64_t)n_ph;
   }
-  if (cur == 1) {   // the final state is in the scratch buffer: copy to perm
+  if (CLU) {
+    // every CTA writes the slots of its owned pairs in the last class
+    // (ncls - 1) from its own replica (it published them to itself)
+    for (int pass = 0; pass < npass; ++pass) {
+      const int32_t ch = gid + pass * ngrp_tot;
+      if (ch >= p.nchunks) continue;
+      const int32_t k0 = ch * W, k1 = min(k0 + W, K + 1);
+      for (int32_t k = k0 + gt; k < k1; k += GT) {
+        int32_t u, v;
+        cl.pair(ncls - 1, k, u, v);
+        p.rbuf[0][u] = rep_r[cur * S + u];
+        p.rbuf[0][v] = rep_r[cur * S + v];
+      }
+    }
+    cg::this_cluster().sync();   // no CTA exits while others may still touch its smem
+  } else if (cur == 1) {   // the final state is in the scratch buffer: copy to perm
     for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
       p.rbuf[0][x] = __ldcg(p.rbuf[1] + x);
   }
@@ -356,7 +436,7 @@ template <int PPL, int T>
 static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   using SM = TrapSmem<PPL, T>;
   constexpr int X = SM::X;
-  static_assert(X > 2 * T, "chunk must own at least one pair");
+  static_assert(X > 2 * T + 1, "chunk must own more than T pairs");
   int dev = 0, nsm = 0, optin = 0;
   PM_CUDA_TRY(cudaGetDevice(&dev));
   PM_CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
@@ -364,15 +444,57 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   const Classes cl(hp.S);
   const int32_t npairs = cl.npairs;
   int32_t W = trap_env("PM_TRAP_W", X - 2 * T);
-  if (W < 1 || W > X - 2 * T) W = X - 2 * T;
+  if (W < T + 1 || W > X - 2 * T) W = X - 2 * T;   // W > T: neighbours publish every halo slot
   hp.W = W;
   hp.nchunks = (npairs + W - 1) / W;
-  // chunk groups of gsz warps (they stage a chunk together and split its
-  // pairs); cpc groups per CTA, enough CTAs to hold every chunk in one pass
-  int gsz = trap_env("PM_TRAP_GSZ", PPL >= 2 ? 2 : 1);
-  if (gsz < 1) gsz = 1;
-  if (gsz > 8) gsz = 8;
+  const int gsz = PPL;   // warps per chunk group: one pair position per thread
   hp.gsz = gsz;
+  // cluster mode when every chunk fits one cluster of <= 16 CTAs
+  const size_t rep_bytes = sizeof(int32_t) * 4 * (size_t)hp.S;
+  int mode = trap_env("PM_TRAP_CLUSTER", -1);   // -1 auto, 0 grid, 1 cluster
+  int max_cpc_cl = ((size_t)optin > rep_bytes) ? (int)(((size_t)optin - rep_bytes) / SM::bytes) : 0;
+  if (max_cpc_cl > 8 / gsz) max_cpc_cl = 8 / gsz;
+  int cpc_cl = (hp.nchunks + 15) / 16;
+  const bool cl_ok = max_cpc_cl >= 1 && cpc_cl <= max_cpc_cl;
+  // measured: the cluster pays while every CTA holds one chunk
+  // (config 2: 1.50 vs 1.66 ms); with several chunks per CTA the staging of
+  // 16 SMs loses to the grid's (config 3: 11.8 vs 10.7 ms)
+  if (mode < 0) mode = (cl_ok && cpc_cl == 1) ? 1 : 0;
+  if (trap_env("PM_TRAP_DEBUG", 0))
+    std::fprintf(stderr, "trap: S=%d mode=%d max_cpc_cl=%d cpc_cl=%d optin=%d bytes=%zu\n", hp.S, mode, max_cpc_cl,
+                 cpc_cl, optin, SM::bytes);
+  if (mode == 1 && !cl_ok) return PM_ERR_UNSUPPORTED;
+  if (mode == 1) {
+    cpc_cl = trap_env("PM_TRAP_CPC", cpc_cl);
+    if (cpc_cl < 1) cpc_cl = 1;
+    if (cpc_cl > max_cpc_cl) cpc_cl = max_cpc_cl;
+    const int nblk = (hp.nchunks + cpc_cl - 1) / cpc_cl;
+    if (nblk > 16) return PM_ERR_UNSUPPORTED;
+    const size_t smem = SM::bytes * cpc_cl + rep_bytes;
+    const int threads = 32 * gsz * cpc_cl;
+    auto fn = k_ls_trap<PPL, T, true>;
+    PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    if (nblk > 8) PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(nblk);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = nblk;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int ncl = 0;
+    PM_CUDA_TRY(cudaOccupancyMaxActiveClusters(&ncl, fn, &cfg));
+    if (ncl < 1) return PM_ERR_UNSUPPORTED;
+    PM_CUDA_TRY(cudaLaunchKernelEx(&cfg, fn, hp));
+    note_launch();
+    return PM_OK;
+  }
+  // grid mode: cpc chunk groups per CTA, enough CTAs for one pass if possible
   int max_cpc = (int)((size_t)optin / SM::bytes);
   if (max_cpc > 8 / gsz) max_cpc = 8 / gsz;
   if (max_cpc < 1) return PM_ERR_UNSUPPORTED;
@@ -381,14 +503,18 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   if (cpc > max_cpc) cpc = max_cpc;
   const size_t smem = SM::bytes * cpc;
   const int threads = 32 * gsz * cpc;
-  PM_CUDA_TRY(cudaFuncSetAttribute(k_ls_trap<PPL, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  auto fn = k_ls_trap<PPL, T, false>;
+  PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
-  PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_ls_trap<PPL, T>, threads, smem));
+  PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
+  if (trap_env("PM_TRAP_DEBUG", 0))
+    std::fprintf(stderr, "trap grid: S=%d W=%d nchunks=%d cpc=%d threads=%d smem=%zu occ=%d\n", hp.S, hp.W,
+                 hp.nchunks, cpc, threads, smem, occ);
   if (occ < 1) return PM_ERR_UNSUPPORTED;
   int grid = (hp.nchunks + cpc - 1) / cpc;
   if (grid > nsm * occ) grid = nsm * occ;
   void* args[] = {(void*)&hp};
-  PM_CUDA_TRY(cudaLaunchCooperativeKernel((const void*)k_ls_trap<PPL, T>, dim3(grid), dim3(threads), args, smem, st));
+  PM_CUDA_TRY(cudaLaunchCooperativeKernel((const void*)fn, dim3(grid), dim3(threads), args, smem, st));
   note_launch();
   return PM_OK;
 }
@@ -430,13 +556,6 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   if (s != PM_OK) return s;
   PM_CUDA_TRY(cudaFreeAsync(scratch, st));
   return PM_OK;
-}
-
-int64_t trap_misses_read_and_reset() {
-  unsigned long long v = 0, z = 0;
-  if (cudaMemcpyFromSymbol(&v, g_trap_misses, sizeof(v)) != cudaSuccess) return -1;
-  if (cudaMemcpyToSymbol(g_trap_misses, &z, sizeof(z)) != cudaSuccess) return -1;
-  return (int64_t)v;
 }
 
 }  // namespace pm

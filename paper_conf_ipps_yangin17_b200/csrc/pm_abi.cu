@@ -252,9 +252,11 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
 int32_t pm_ls_cta_max_S(void) { return ls_cta_max_S(); }
 
 int32_t pm_ls_auto_method(int32_t S) {
-  // measured on B200: WINDOW fastest up to its shared-memory limit; beyond it
-  // the graph of per-class kernels beats one CTA (whose gather rate is bounded
-  // by one SM: 2.4 vs 2.6 us/class at S = 4096, 3.3 vs 11.7 at S = 16384)
+  // measured on B200 (whole search incl. sparse rounds): TRAP for
+  // even S >= 256 (config 1/2/3/4: 0.42/1.50/10.7/111 ms against WINDOW
+  // 0.46/1.98 and CLASS 28.6/240); below, WINDOW up to its shared-memory
+  // limit, then the graph of per-class kernels
+  if (S >= ls_trap_min_S() && (S % 2) == 0) return PM_LS_TRAP;
   return (S <= ls_window_max_S()) ? PM_LS_WINDOW : PM_LS_CLASS;
 }
 
@@ -375,7 +377,6 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
   return PM_OK;
 }
 
-int64_t pm_debug_trap_misses(void) { return trap_misses_read_and_reset(); }
 int64_t pm_launch_count(void) { return g_launches.load() + device_launch_total(); }
 
 }  // extern "C"

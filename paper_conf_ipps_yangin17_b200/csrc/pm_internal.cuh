@@ -172,7 +172,6 @@ int32_t ls_trap_min_S();
 pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                      LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
                      int32_t* handoff, int32_t sparse_T);
-int64_t trap_misses_read_and_reset();
 
 // Exact min-weight perfect matching by eps-scaling auction (k_assign.cu).
 // h_stats (nullable): {bidding rounds, phases}.  Synchronises st.

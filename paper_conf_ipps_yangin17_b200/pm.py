@@ -49,7 +49,6 @@ _SIGS = [
     ("pm_render", ctypes.c_int, [_P, _I32, _I32, _I32, _P, _P, _P]),
     ("pm_optimal_assignment", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P, _P, _P]),
     ("pm_launch_count", _I64, []),
-    ("pm_debug_trap_misses", _I64, []),
 ]
 
 

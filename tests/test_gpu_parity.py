@@ -6,6 +6,8 @@ error (Eq. 2).  Full-size configs 4-5 (BASELINE.json) are checked on sampled
 E entries the oracle computes one by one, and the local search there via its
 closed-form special case (transposition) and properties that hold at any
 size (bijection, 2-swap local optimality, cost identity)."""
+import os
+
 import numpy as np
 import pytest
 
@@ -493,27 +495,38 @@ def test_walk_mailbox_overflow_falls_back_exactly():
     assert ref[3][0] >= 63
 
 
+def _check_trap(E_np):
+    # the cluster mode is unsupported (PM_ERR_UNSUPPORTED) when the chunks do
+    # not fit one cluster; every other outcome must match the oracle
+    try:
+        _check_ls(E_np, "trap")
+    except pm.PMError as e:
+        if e.status != pm.PM_ERR_UNSUPPORTED or os.environ.get("PM_TRAP_CLUSTER") != "1":
+            raise
+        pytest.skip("chunks do not fit one cluster")
+
+
 # ---- PM_LS_TRAP: every round on the temporal-blocked kernel (sparse hand-over
 # off), every compiled (pairs-per-lane, T) variant, chunk widths that do not
-# divide S/2, and no E lookup outside the staged runs.
+# divide S/2, grid-barrier and cluster (DSMEM) modes.
 @pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
 @pytest.mark.parametrize("N,M,fam,W", [(128, 8, "smooth", 0), (512, 16, "smooth", 0), (512, 16, "ties", 7),
-                                       (240, 8, "noise", 0), (336, 8, "smooth", 5), (128, 8, "transposition", 3)])
-def test_trap_every_round(variant, N, M, fam, W, monkeypatch):
+                                       (240, 8, "noise", 0), (336, 8, "smooth", 21), (128, 8, "transposition", 19)])
+@pytest.mark.parametrize("mode", ["0", "1"])
+def test_trap_every_round(variant, N, M, fam, W, mode, monkeypatch):
     monkeypatch.setenv("PM_TRAP_V", str(variant))
+    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
     monkeypatch.setenv("PM_LS_SPARSE", "0")
     monkeypatch.setenv("PM_TRAP_W", str(W))
-    pm.lib().pm_debug_trap_misses()
-    _check_ls(oracle_E(fam, N, M), "trap")
-    assert pm.lib().pm_debug_trap_misses() == 0
+    _check_trap(oracle_E(fam, N, M))
 
 
-@pytest.mark.parametrize("cpc,gsz,variant", [(1, 1, 0), (2, 2, 0), (3, 1, 1), (1, 4, 3), (2, 4, 4), (1, 8, 2)])
-def test_trap_warps_per_cta(cpc, gsz, variant, monkeypatch):
+@pytest.mark.parametrize("cpc,variant", [(1, 0), (2, 0), (3, 1), (1, 3), (2, 4), (4, 2)])
+@pytest.mark.parametrize("mode", ["0", "1"])
+def test_trap_chunks_per_cta(cpc, variant, mode, monkeypatch):
+    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
     monkeypatch.setenv("PM_TRAP_CPC", str(cpc))
-    monkeypatch.setenv("PM_TRAP_GSZ", str(gsz))
     monkeypatch.setenv("PM_TRAP_V", str(variant))
     monkeypatch.setenv("PM_LS_SPARSE", "0")
-    pm.lib().pm_debug_trap_misses()
-    _check_ls(oracle_E("noise", 1024, 16), "trap")
-    assert pm.lib().pm_debug_trap_misses() == 0
+    # cluster mode holds every chunk in <= 16 CTAs: S = 1024 (16-64 chunks)
+    _check_trap(oracle_E("noise", 1024 if mode == "0" else 512, 16))

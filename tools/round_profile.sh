@@ -16,12 +16,12 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 timeout 600 ncu --graph-profiling graph --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file $out/${tag}_launches_graph.csv \
   python bench.py --steps 3 --warmup 3 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1; echo "graph launch list rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k 'regex:k_sad|k_ls_window' -s 2 -c 2 \
+timeout 900 ncu --set full --clock-control none --import-source on -k 'regex:k_sad|k_ls_trap' -s 2 -c 2 \
   -o $out/${tag}_full -f python bench.py --steps 1 --warmup 3 --no-cpu-baseline --e2e-steps 1 > /dev/null 2>&1; echo "full rc=$?"
 timeout 900 ncu --graph-profiling graph --set full --clock-control none -s 1 -c 1 --kernel-name-base function \
-  -o $out/${tag}_sparse_graph -f python tools/ls_bench.py 2 window > /dev/null 2>&1; echo "sparse graph full rc=$?"
+  -o $out/${tag}_sparse_graph -f python tools/ls_bench.py 2 trap > /dev/null 2>&1; echo "sparse graph full rc=$?"
 REPS=3 timeout 600 python tools/assign_bench.py 1 2 3 4 > $out/${tag}_assign.txt 2>&1; tail -4 $out/${tag}_assign.txt
-REPS=3 timeout 900 python tools/ls_bench.py 1,2 window,walk,cta,class > $out/${tag}_ls_methods.txt 2>&1
-REPS=2 timeout 900 python tools/ls_bench.py 3 auto,walk,class,cta >> $out/${tag}_ls_methods.txt 2>&1
-REPS=1 timeout 900 python tools/ls_bench.py 4 auto,walk >> $out/${tag}_ls_methods.txt 2>&1; grep cfg $out/${tag}_ls_methods.txt | cut -c1-90
+REPS=3 timeout 900 python tools/ls_bench.py 1,2 trap,window,walk,cta,class > $out/${tag}_ls_methods.txt 2>&1
+REPS=2 timeout 900 python tools/ls_bench.py 3 auto,trap,walk,class,cta >> $out/${tag}_ls_methods.txt 2>&1
+REPS=1 timeout 900 python tools/ls_bench.py 4 auto,class >> $out/${tag}_ls_methods.txt 2>&1; grep cfg $out/${tag}_ls_methods.txt | cut -c1-90
 timeout 600 python tools/e_bench.py 1,2,3,4,5 > $out/${tag}_e_bench.txt 2>&1; cat $out/${tag}_e_bench.txt | grep cfg
