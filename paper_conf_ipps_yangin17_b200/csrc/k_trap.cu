@@ -57,6 +57,7 @@ struct TrapParams {
   int32_t S, max_rounds, max_log, sparse_T;
   int32_t W, nchunks;
   int32_t gsz;                 // warps per chunk group (= PPL)
+  int32_t vec;                 // 16-byte staging allowed (PM_TRAP_VEC, default 1)
   int32_t prof;                // PM_TRAP_PROF: CTA 0 thread 0 phase timers -> per_round[192..195]
   unsigned int* bar;           // grid barrier counter (zeroed before launch)
   unsigned long long* rsw;     // [3] swaps per round, rotating (grid mode)
@@ -70,12 +71,14 @@ template <int PPL, int T>
 struct TrapSmem {
   static constexpr int X = 32 * PPL;        // pairs of an extended range
   static constexpr int L = 2 * X;           // slots (= tiles) of an extended range
-  // staged row of local tile i: run0 [R0, R0+T+1) = E[g][p0 + 2j], run1
-  // [R1, R1+T+1) = E[g][s0 + 2j], E[g][S-1] at CL; odd stride (banks)
-  static constexpr int R0 = 0, R1 = T + 1, CL = 2 * T + 2;
-  static constexpr int RS = 2 * T + 3;
+  // staged row of local tile i: span0 [0, SP) holds E[g][(p0 & ~3) + q] and
+  // span1 [SP, 2SP) E[g][(s0 & ~3) + q] (16-byte copies; the runs p0 + 2j,
+  // s0 + 2j, j <= T, are their entries (p0 & 3) + 2j), E[g][S-1] at CL
+  static constexpr int SP = (2 * T + 4 + 3) / 4 * 4;
+  static constexpr int CL = 2 * SP;
+  static constexpr int RS = 2 * SP + 4;
   static constexpr int NC = 2 * T + 2;      // pair-0 light-cone tiles (at most)
-  static constexpr int NU = 2 * T + 3;      // their runU = E[g][u0 + z], z <= 2T+1 (odd stride)
+  static constexpr int NU = (2 * T + 2 + 3 + 3) / 4 * 4;   // their span of E[g][u0 + z], z <= 2T+1
   static constexpr int UOFF = L * RS;       // cone rows follow the rows (one index space)
   static constexpr int ints = (L * (4 + 1 + RS) + NC * NU + 3) / 4 * 4;   // int4 state + g + rows + cone rows
   static constexpr size_t bytes = sizeof(int32_t) * (size_t)ints;
@@ -95,6 +98,25 @@ __device__ __forceinline__ unsigned long long gtimer() {
 __device__ __forceinline__ void cp_async4(int32_t* dst, const int32_t* src) {
   const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(s), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(int32_t* dst, const int32_t* src) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s), "l"(src) : "memory");
+}
+// E[row][first .. first + n) (n = 4 * pieces) into dst (16-byte aligned): one
+// 16-byte copy per piece when the span is in the regular columns and rows are
+// 16-byte aligned, else entry by entry with the column taken mod m.
+__device__ __forceinline__ void stage_span(int32_t* dst, const int32_t* row, int32_t first, int32_t n, int32_t m,
+                                           bool vec) {
+  if (vec && first + n <= m) {
+    for (int32_t q = 0; q < n; q += 4) cp_async16(dst + q, row + first + q);
+  } else {
+    for (int32_t q = 0; q < n; ++q) {
+      int32_t y = first + q;
+      y = y >= m ? y - m : y;
+      cp_async4(dst + q, row + y);
+    }
+  }
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
@@ -152,7 +174,7 @@ template <int PPL, int T, typename Src>
 __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_t k1, int32_t c0, int32_t u0,
                                           const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
                                           int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
-                                          unsigned long long* tprof) {
+                                          bool vec, unsigned long long* tprof) {
   using SM = TrapSmem<PPL, T>;
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
@@ -167,32 +189,17 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     s_g[j] = g;
     const bool fx = (x == S - 1);
     const int32_t ci = C.cone(j);
-    s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU, 0)
-                 : make_int4(j | (1 << 16), d, j * RS + SM::R0, j * RS + SM::R1 + 1);
-    const int32_t* row = E + (int64_t)g * ld;
-    int32_t* dst = s_E + j * RS;
-    // run0: E[g][p0 + 2c], run1: E[g][x + 2c] (c <= T), E[g][S-1];
     // p0 = partner in class c0 (the fixed tile's runs are unused)
     const int32_t p0 = fx ? u0 : wrap_m(2 * c0 + 1 - x, m);
     const int32_t s0 = fx ? u0 : x;
-#pragma unroll
-    for (int32_t c = 0; c <= T; ++c) {
-      int32_t y0 = p0 + 2 * c, y1 = s0 + 2 * c;
-      y0 = y0 >= m ? y0 - m : y0;
-      y1 = y1 >= m ? y1 - m : y1;
-      cp_async4(dst + SM::R0 + c, row + y0);
-      cp_async4(dst + SM::R1 + c, row + y1);
-    }
+    s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
+                 : make_int4(j | (2 << 16), d, j * RS + (p0 & 3), j * RS + SM::SP + (s0 & 3) + 2);
+    const int32_t* row = E + (int64_t)g * ld;
+    int32_t* dst = s_E + j * RS;
+    stage_span(dst, row, p0 & ~3, SM::SP, m, vec);
+    stage_span(dst + SM::SP, row, s0 & ~3, SM::SP, m, vec);
     cp_async4(dst + SM::CL, row + (S - 1));
-    if (ci >= 0) {
-      int32_t* du = s_U + ci * SM::NU;
-#pragma unroll
-      for (int32_t z = 0; z < 2 * T + 2; ++z) {
-        int32_t y = u0 + z;
-        y = y >= m ? y - m : y;
-        cp_async4(du + z, row + y);
-      }
-    }
+    if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, vec);
   }
   cp_async_wait_all();
   group_sync(bar_id, GT);
@@ -215,9 +222,9 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       int4 nA = sw ? make_int4(B.x, e_bu, B.w, B.z + ib) : make_int4(A.x, A.y, A.z + ia, A.w);
       int4 nB = sw ? make_int4(A.x, e_av, A.w, A.z + ia) : make_int4(B.x, B.y, B.z + ib, B.w);
       if (k == 0 && sw) {   // B leaves S-1 for slot u0+t (next partner u0+t+2), A enters S-1
-        const int32_t rb = SM::UOFF + C.cone(B.x & 0xffff) * SM::NU + t + 2;
+        const int32_t rb = SM::UOFF + C.cone(B.x & 0xffff) * SM::NU + (u0 & 3) + t + 2;
         nA = make_int4((B.x & 0xffff) | (2 << 16), e_bu, rb, rb);
-        nB = make_int4((A.x & 0xffff) | (1 << 16), e_av, SM::UOFF + C.cone(A.x & 0xffff) * SM::NU + t + 1, 0);
+        nB = make_int4((A.x & 0xffff) | (1 << 16), e_av, SM::UOFF + C.cone(A.x & 0xffff) * SM::NU + (u0 & 3) + t + 1, 0);
       }
       s_st[j1] = nA;
       s_st[j2] = nB;
@@ -252,6 +259,7 @@ k_ls_trap(const TrapParams p) {
 
   const int32_t* __restrict__ E = p.E;
   const int64_t ld = p.ldE;
+  const bool vec = p.vec && ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);   // 16-byte row pieces
   const Classes cl(S);
   const int32_t m = cl.m, H = cl.half, K = cl.npairs - 1, ncls = cl.ncls;
   const int32_t W = p.W;
@@ -311,13 +319,13 @@ k_ls_trap(const TrapParams p) {
             const int32_t* rd = rep_d + cur * S;
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { g = rr[x]; d = rd[x]; },
-                                       s_st, s_g, s_E, gt, 1 + grp, prof ? &t_st : nullptr);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
           } else {
             const int32_t* __restrict__ rc = cur ? p.rbuf[1] : p.rbuf[0];
             const int32_t* __restrict__ dc = cur ? p.dbuf[1] : p.dbuf[0];
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
-                                       s_st, s_g, s_E, gt, 1 + grp, prof ? &t_st : nullptr);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
           // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
@@ -544,6 +552,10 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.launches = device_launch_counter();
   if (!hp.launches) return PM_ERR_CUDA;
   hp.prof = trap_env("PM_TRAP_PROF", 0);
+  // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
+  // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
+  // used runs win (config 4: 5.0 vs 10.8 us)
+  hp.vec = trap_env("PM_TRAP_VEC", (int64_t)S * ldE * 4 <= (96ll << 20) ? 1 : 0);
   const int32_t variant = trap_env("PM_TRAP_V", 0);
   pm_status_t s;
   switch (variant) {

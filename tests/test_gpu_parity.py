@@ -521,7 +521,7 @@ def test_trap_every_round(variant, N, M, fam, W, mode, monkeypatch):
     _check_trap(oracle_E(fam, N, M))
 
 
-@pytest.mark.parametrize("cpc,variant", [(1, 0), (2, 0), (3, 1), (1, 3), (2, 4), (4, 2)])
+@pytest.mark.parametrize("cpc,variant", [(1, 0), (2, 0), (3, 1), (1, 3), (2, 4), (4, 2), (8, 1)])
 @pytest.mark.parametrize("mode", ["0", "1"])
 def test_trap_chunks_per_cta(cpc, variant, mode, monkeypatch):
     monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
@@ -530,3 +530,27 @@ def test_trap_chunks_per_cta(cpc, variant, mode, monkeypatch):
     monkeypatch.setenv("PM_LS_SPARSE", "0")
     # cluster mode holds every chunk in <= 16 CTAs: S = 1024 (16-64 chunks)
     _check_trap(oracle_E("noise", 1024 if mode == "0" else 512, 16))
+
+
+@pytest.mark.parametrize("method", ["trap", "class", "window"])
+def test_local_search_padded_leading_dimension(method):
+    # E as the left S columns of a wider matrix (ld_E = S + 3): TRAP's
+    # 16-byte row pieces need ld_E % 4 == 0 and take the entry-wise path here
+    E_np = oracle_E("smooth", 512, 16)
+    S = E_np.shape[0]
+    ref = oracle.local_search(E_np)
+    big = torch.full((S, S + 3), -1, dtype=torch.int32, device=DEV)
+    big[:, :S] = dev(E_np)
+    out, rounds, swaps, per, st = pm.local_search(big[:, :S], method=method)
+    assert (out.cpu().numpy() == ref[0]).all()
+    assert (rounds, swaps) == (ref[1], ref[2])
+
+
+@pytest.mark.parametrize("variant,mode,vec", [("0", "0", "1"), ("0", "0", "0"), ("1", "1", "1"), ("3", "0", "1")])
+def test_trap_every_round_config3(variant, mode, vec, monkeypatch):
+    # S = 4096 with P = 768: pair-0 swaps at every u0 mod 4 (the 16-byte span offsets)
+    monkeypatch.setenv("PM_TRAP_V", variant)
+    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
+    monkeypatch.setenv("PM_TRAP_VEC", vec)
+    monkeypatch.setenv("PM_LS_SPARSE", "0")
+    _check_trap(oracle_E("smooth", 1024, 16))
