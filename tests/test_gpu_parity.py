@@ -255,6 +255,28 @@ def test_local_search_config4_properties_and_closed_form():
     assert pm.cost(E, perm) == int(E[perm.long(), torch.arange(16384, device=DEV)].to(torch.int64).sum())
 
 
+def test_local_search_config5_properties_and_closed_form():
+    # n = 65536 (E = 16 GiB): transposition closed form (1 swap, 2 rounds,
+    # cost 0) and, on the smooth family, bijection + 2-opt + cost identity
+    I, T = pair("transposition", 4096, 16)
+    E = pm.error_matrix(dev(I), dev(T), 16)
+    moved = torch.nonzero(torch.diagonal(E)).flatten().cpu().numpy()
+    assert len(moved) == 2
+    perm, rounds, swaps, per, st = pm.local_search(E)
+    expect = np.arange(65536)
+    expect[moved[0]], expect[moved[1]] = moved[1], moved[0]
+    assert (perm.cpu().numpy() == expect).all() and (rounds, swaps) == (2, 1)
+    assert pm.cost(E, perm) == 0
+    del E
+    I, T = pair("smooth", 4096, 16)
+    E = pm.error_matrix(dev(I), dev(T), 16)
+    perm, rounds, swaps, per, st = pm.local_search(E)
+    assert sorted(perm.cpu().numpy().tolist()) == list(range(65536))
+    assert per[-1] == 0 and per.sum() == swaps
+    assert _two_opt_gpu(E, perm)
+    assert pm.cost(E, perm) == int(E[perm.long(), torch.arange(65536, device=DEV)].to(torch.int64).sum())
+
+
 # ------------------------------------------------------------------ Eq. (2) -
 @pytest.mark.parametrize("N,M,C", [(128, 8, 3), (512, 16, 3), (90, 10, 3)])
 def test_cost_parity(N, M, C):
