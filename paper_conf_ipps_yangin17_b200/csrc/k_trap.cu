@@ -140,6 +140,33 @@ __device__ __forceinline__ void grid_barrier(unsigned int* bar, unsigned int tar
   __syncthreads();
 }
 
+// ---- cluster mode: DSMEM stores that complete on the receiver's mbarrier ----
+__device__ __forceinline__ uint32_t smem_u32(const void* ptr) { return (uint32_t)__cvta_generic_to_shared(ptr); }
+__device__ __forceinline__ uint32_t cluster_addr(uint32_t a, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void st_async_v2(uint32_t raddr, int32_t x, int32_t y, uint32_t rmbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.s32 [%0], {%1, %2}, [%3];" ::"r"(raddr),
+               "r"(x), "r"(y), "r"(rmbar)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_init(uint64_t* mbar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(mbar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* mbar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mbar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t* mbar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred P1;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P1, [%0], %1;\n"
+      " @!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(mbar)),
+      "r"(parity)
+      : "memory");
+}
+
 // Local slot j of a chunk's extended range [a, b): j < nA -> slot u0 + a + j
 // (first slots), j < nA + nB -> slot u0 - (a2 + j - nA) (second slots),
 // j = nA + nB -> S - 1 (only when a == 0).  Pair k at step t (class c0 + t)
@@ -204,16 +231,23 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
   cp_async_wait_all();
   group_sync(bar_id, GT);
   unsigned long long t0 = tprof ? gtimer() : 0;
-  // ---- Tp classes on the extended range: thread gt takes pair a + gt ----
+  // ---- Tp classes on the extended range: thread gt takes pair k = a + gt,
+  // valid while t <= tmax (the trapezoid); its local slots are linear in t ----
   int mysw = 0;
   const int32_t k = C.a + gt;
   const bool own = (k >= k0 && k < k1);
+  int32_t tmax = -1;
+  if (k < C.b) {
+    tmax = Tp - 1;
+    if (!low) tmax = min(tmax, k - C.a);
+    if (C.b != K + 1) tmax = min(tmax, C.b - 1 - k);
+  }
+  const int32_t tk = K - k, b1 = k - C.a, c1 = C.nA + m - C.a2 - k;   // j1 = t <= tk ? b1 + t : c1 - t
+  const int32_t b2 = -k - C.a, c2 = C.nA + k - C.a2;                   // j2 = t >= k ? b2 + t : c2 - t
   for (int32_t t = 0; t < Tp; ++t) {
-    const int32_t lo = low ? 0 : C.a + t;
-    const int32_t hi = (C.b == K + 1) ? K + 1 : C.b - t;
-    if (k >= lo && k < hi) {
-      int32_t j1, j2;
-      C.local_slots(t, k, j1, j2);
+    if (t <= tmax) {
+      const int32_t j1 = (t <= tk) ? b1 + t : c1 - t;
+      const int32_t j2 = (k == 0) ? Lc - 1 : ((t >= k) ? b2 + t : c2 - t);
       const int4 A = s_st[j1], B = s_st[j2];
       const int32_t e_bu = s_E[B.z];
       const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z];
@@ -251,11 +285,12 @@ k_ls_trap(const TrapParams p) {
   int32_t* s_g = ws + 4 * L;
   int32_t* s_E = s_g + L;
   const int32_t S = p.S;
-  // cluster mode: replicas of r and d, ping-pong [2][S] each
-  int32_t* rep_r = sm + (size_t)cpc * SM::ints;
-  int32_t* rep_d = rep_r + 2 * S;
+  // cluster mode (one chunk per CTA): replica {r, d} of every slot, ping-pong
+  // [2][S]; mbar[b] completes when the neighbours' slots for buffer b landed
+  int2* rep = reinterpret_cast<int2*>(sm + (size_t)cpc * SM::ints);
   __shared__ int32_t s_cta_sw;
   __shared__ unsigned long long s_rs, s_rsw[3];
+  __shared__ __align__(8) uint64_t s_mbar[2];
 
   const int32_t* __restrict__ E = p.E;
   const int64_t ld = p.ldE;
@@ -273,11 +308,22 @@ k_ls_trap(const TrapParams p) {
 
   if (threadIdx.x == 0) { s_cta_sw = 0; s_rsw[0] = s_rsw[1] = s_rsw[2] = 0ull; }
   // d[x] = E[r[x]][x] (the maintained diagonal)
+  // bytes of published slots this CTA receives per phase: chunks ch-1..ch+1
+  // each send 2 slots x 8 bytes per owned pair
+  uint32_t rx_bytes = 0;
   if (CLU) {
+    for (int dch = -1; dch <= 1; ++dch) {
+      const int32_t c2 = (int32_t)blockIdx.x + dch;
+      if (c2 >= 0 && c2 < p.nchunks) rx_bytes += 16u * (uint32_t)(min((c2 + 1) * W, K + 1) - c2 * W);
+    }
     for (int32_t x = threadIdx.x; x < S; x += blockDim.x) {
       const int32_t g = __ldcg(p.rbuf[0] + x);
-      rep_r[x] = g;
-      rep_d[x] = __ldg(E + (int64_t)g * ld + x);
+      rep[x] = make_int2(g, __ldg(E + (int64_t)g * ld + x));
+    }
+    if (threadIdx.x == 0) {
+      mbar_init(&s_mbar[0], 1);
+      mbar_init(&s_mbar[1], 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     cg::this_cluster().sync();
   } else {
@@ -291,14 +337,14 @@ k_ls_trap(const TrapParams p) {
   int32_t rounds = 0;
   int64_t total = 0;
   int status = PM_OK;
-  const bool prof = p.prof && blockIdx.x == 0 && threadIdx.x == 0 && p.max_log >= 200;
-  unsigned long long t_ld = 0, t_st = 0, t_bar = 0, n_ph = 0, tq = prof ? gtimer() : 0;
+  // PM_TRAP_PROF = 1: CTA 0, 2: the last CTA, 3: the middle one
+  const unsigned pblk = p.prof == 2 ? nblk - 1 : (p.prof == 3 ? nblk / 2 : 0);
+  const bool prof = p.prof && blockIdx.x == pblk && threadIdx.x == 0 && p.max_log >= 200;
+  unsigned long long t_ld = 0, t_st = 0, t_bar = 0, t_pub = 0, n_ph = 0, tq = prof ? gtimer() : 0;
   const int npass = (p.nchunks + ngrp_tot - 1) / ngrp_tot;
+  uint32_t nph_cl = 0;   // cluster mode: phases completed (mbarrier parity)
   for (;;) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-      if (CLU) s_rsw[(rounds + 1) % 3] = 0ull;
-      else p.rsw[(rounds + 1) % 3] = 0ull;
-    }
+    if (!CLU && blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
       const int32_t u0 = wrap_m(c0 + H, m);
@@ -315,10 +361,9 @@ k_ls_trap(const TrapParams p) {
         C.K = K; C.m = m; C.Tp = Tp;
         if (have) {
           if (CLU) {
-            const int32_t* rr = rep_r + cur * S;
-            const int32_t* rd = rep_d + cur * S;
+            const int2* rr = rep + cur * S;
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
-                                       [&](int32_t x, int32_t& g, int32_t& d) { g = rr[x]; d = rd[x]; },
+                                       [&](int32_t x, int32_t& g, int32_t& d) { const int2 v = rr[x]; g = v.x; d = v.y; },
                                        s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
           } else {
             const int32_t* __restrict__ rc = cur ? p.rbuf[1] : p.rbuf[0];
@@ -339,20 +384,17 @@ k_ls_trap(const TrapParams p) {
               const int32_t g1 = s_g[A.x & 0xffff], g2 = s_g[B.x & 0xffff];
               if (CLU) {
                 // to the replicas of the CTAs of chunks ch-1, ch, ch+1 (every slot of
-                // a chunk's next extended range is published by one of them: W > T)
-                cg::cluster_group cgc = cg::this_cluster();
+                // a chunk's next extended range is published by one of them: W > T),
+                // each store completing on the receiver's mbarrier for that buffer
                 const int nx = cur ^ 1;
-                int lastb = -1;
+                const uint32_t a1 = smem_u32(rep + nx * S + x1), a2 = smem_u32(rep + nx * S + x2);
+                const uint32_t am = smem_u32(&s_mbar[nx]);
                 for (int dch = -1; dch <= 1; ++dch) {
                   const int32_t c2 = ch + dch;
                   if (c2 < 0 || c2 >= p.nchunks) continue;
-                  const int blk = c2 / cpc;
-                  if (blk == lastb) continue;
-                  lastb = blk;
-                  int32_t* rr = cgc.map_shared_rank(rep_r, blk) + nx * S;
-                  int32_t* rd = cgc.map_shared_rank(rep_d, blk) + nx * S;
-                  rr[x1] = g1; rd[x1] = A.y;
-                  rr[x2] = g2; rd[x2] = B.y;
+                  const uint32_t rm = cluster_addr(am, c2);
+                  st_async_v2(cluster_addr(a1, c2), g1, A.y, rm);
+                  st_async_v2(cluster_addr(a2, c2), g2, B.y, rm);
                 }
               } else {
                 int32_t* rn = cur ? p.rbuf[0] : p.rbuf[1];
@@ -363,6 +405,7 @@ k_ls_trap(const TrapParams p) {
             }
           }
         }
+        if (prof) { const unsigned long long t = gtimer(); t_pub += t - tq; }
         group_sync(1 + grp, GT);
       }
       // swaps of this phase -> the round counter
@@ -371,13 +414,21 @@ k_ls_trap(const TrapParams p) {
       if ((threadIdx.x & 31) == 0 && mysw) atomicAdd(&s_cta_sw, mysw);
       cur ^= 1;
       __syncthreads();
-      if (threadIdx.x == 0 && s_cta_sw) {
-        if (CLU) atomicAdd(cg::this_cluster().map_shared_rank(&s_rsw[rounds % 3], 0), (unsigned long long)s_cta_sw);
-        else atomicAdd(p.rsw + rounds % 3, (unsigned long long)s_cta_sw);
+      // the CTA's swaps of the round leave the CTA once, before the round's
+      // last barrier: cluster -> its own slot s_rsw[round % 3] (read by every
+      // CTA over DSMEM after the barrier), grid -> one global atomic
+      if (c0 + T >= ncls && threadIdx.x == 0) {
+        if (CLU) s_rsw[rounds % 3] = (unsigned long long)s_cta_sw;
+        else if (s_cta_sw) atomicAdd(p.rsw + rounds % 3, (unsigned long long)s_cta_sw);
         s_cta_sw = 0;
       }
       if (CLU) {
-        cg::this_cluster().sync();
+        // wait for the neighbours' slots of the next phase (buffer cur, now);
+        // mbar[b] is used every other phase: parity = its use count & 1
+        if (threadIdx.x == 0) mbar_arrive_expect_tx(&s_mbar[cur], rx_bytes);
+        mbar_wait_parity(&s_mbar[cur], (uint32_t)(nph_cl >> 1) & 1u);
+        ++nph_cl;
+        if (c0 + T >= ncls) cg::this_cluster().sync();   // round end: every CTA's s_rsw slot is set
       } else {
         bar_target += nblk;
         grid_barrier(p.bar, bar_target);
@@ -385,17 +436,23 @@ k_ls_trap(const TrapParams p) {
       if (prof) { const unsigned long long t = gtimer(); t_bar += t - tq; tq = t; ++n_ph; }
     }
     // round end (Alg. 2 lines 10-11)
-    if (threadIdx.x == 0) {
-      if (CLU) s_rs = *cg::this_cluster().map_shared_rank(&s_rsw[rounds % 3], 0);
-      else s_rs = *((volatile unsigned long long*)(p.rsw + rounds % 3));
+    if (CLU) {
+      if (threadIdx.x < 32) {
+        unsigned long long v = 0;
+        for (int b = threadIdx.x; b < (int)nblk; b += 32) v += *cg::this_cluster().map_shared_rank(&s_rsw[rounds % 3], b);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (threadIdx.x == 0) s_rs = v;
+      }
+    } else if (threadIdx.x == 0) {
+      s_rs = *((volatile unsigned long long*)(p.rsw + rounds % 3));
     }
     __syncthreads();
     const int64_t rs = (int64_t)s_rs;
     if (blockIdx.x == 0 && threadIdx.x == 0 && rounds < p.max_log) p.per_round[rounds] = rs;
     rounds += 1;
     total += rs;
-    if (CLU) cg::this_cluster().sync();   // CTA 0 resets the next counter only after every read
-    else __syncthreads();
+    __syncthreads();   // (a CTA's s_rsw slot is rewritten three rounds later)
     if (rs == 0) break;
     if (p.max_rounds > 0 && rounds >= p.max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
     if (p.handoff && rs <= p.sparse_T) {
@@ -406,6 +463,7 @@ k_ls_trap(const TrapParams p) {
   if (prof) {
     p.per_round[192] = (int64_t)(t_ld - t_st); p.per_round[193] = (int64_t)t_st;
     p.per_round[194] = (int64_t)t_bar; p.per_round[195] = (int64_t)n_ph;
+    p.per_round[196] = (int64_t)t_pub;
   }
   if (CLU) {
     // every CTA writes the slots of its owned pairs in the last class
@@ -417,8 +475,8 @@ k_ls_trap(const TrapParams p) {
       for (int32_t k = k0 + gt; k < k1; k += GT) {
         int32_t u, v;
         cl.pair(ncls - 1, k, u, v);
-        p.rbuf[0][u] = rep_r[cur * S + u];
-        p.rbuf[0][v] = rep_r[cur * S + v];
+        p.rbuf[0][u] = rep[cur * S + u].x;
+        p.rbuf[0][v] = rep[cur * S + v].x;
       }
     }
     cg::this_cluster().sync();   // no CTA exits while others may still touch its smem
@@ -462,21 +520,19 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   int mode = trap_env("PM_TRAP_CLUSTER", -1);   // -1 auto, 0 grid, 1 cluster
   int max_cpc_cl = ((size_t)optin > rep_bytes) ? (int)(((size_t)optin - rep_bytes) / SM::bytes) : 0;
   if (max_cpc_cl > 8 / gsz) max_cpc_cl = 8 / gsz;
-  int cpc_cl = (hp.nchunks + 15) / 16;
-  const bool cl_ok = max_cpc_cl >= 1 && cpc_cl <= max_cpc_cl;
+  // (cluster mode: one chunk per CTA, its neighbours' CTAs = chunks ch +- 1)
+  const bool cl_ok = max_cpc_cl >= 1 && hp.nchunks <= 16;
   // measured: the cluster pays while every CTA holds one chunk
   // (config 2: 1.50 vs 1.66 ms); with several chunks per CTA the staging of
   // 16 SMs loses to the grid's (config 3: 11.8 vs 10.7 ms)
-  if (mode < 0) mode = (cl_ok && cpc_cl == 1) ? 1 : 0;
+  if (mode < 0) mode = cl_ok ? 1 : 0;
   if (trap_env("PM_TRAP_DEBUG", 0))
-    std::fprintf(stderr, "trap: S=%d mode=%d max_cpc_cl=%d cpc_cl=%d optin=%d bytes=%zu\n", hp.S, mode, max_cpc_cl,
-                 cpc_cl, optin, SM::bytes);
+    std::fprintf(stderr, "trap: S=%d mode=%d max_cpc_cl=%d nchunks=%d optin=%d bytes=%zu\n", hp.S, mode, max_cpc_cl,
+                 hp.nchunks, optin, SM::bytes);
   if (mode == 1 && !cl_ok) return PM_ERR_UNSUPPORTED;
   if (mode == 1) {
-    cpc_cl = trap_env("PM_TRAP_CPC", cpc_cl);
-    if (cpc_cl < 1) cpc_cl = 1;
-    if (cpc_cl > max_cpc_cl) cpc_cl = max_cpc_cl;
-    const int nblk = (hp.nchunks + cpc_cl - 1) / cpc_cl;
+    const int cpc_cl = 1;
+    const int nblk = hp.nchunks;
     if (nblk > 16) return PM_ERR_UNSUPPORTED;
     const size_t smem = SM::bytes * cpc_cl + rep_bytes;
     const int threads = 32 * gsz * cpc_cl;

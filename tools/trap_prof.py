@@ -24,7 +24,7 @@ for cfg in cfgs:
         r, sw = ctypes.c_int32(0), ctypes.c_int64(0)
         st = pm.lib().pm_local_search_ex(E.data_ptr(), E.stride(0), S, perm.data_ptr(), 0, pm.METHODS["trap"],
                                          ctypes.byref(r), ctypes.byref(sw), per.ctypes.data, 256, None)
-    ld, stp, bar, nph = per[192:196]
+    ld, stp, bar, nph, pub = per[192:197]
     nph = max(int(nph), 1)
     print(f"cfg{cfg} S={S} st={st} rounds={r.value} phases={nph} per phase: stage {ld/nph:.0f} ns, "
-          f"steps {stp/nph:.0f} ns, writeback+barrier {bar/nph:.0f} ns; total {(ld+stp+bar)/1e6:.3f} ms", flush=True)
+          f"steps {stp/nph:.0f} ns, publish {pub/nph:.0f} ns, publish+barrier {bar/nph:.0f} ns; total {(ld+stp+bar)/1e6:.3f} ms", flush=True)
