@@ -521,7 +521,7 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   int max_cpc_cl = ((size_t)optin > rep_bytes) ? (int)(((size_t)optin - rep_bytes) / SM::bytes) : 0;
   if (max_cpc_cl > 8 / gsz) max_cpc_cl = 8 / gsz;
   // (cluster mode: one chunk per CTA, its neighbours' CTAs = chunks ch +- 1)
-  const bool cl_ok = max_cpc_cl >= 1 && hp.nchunks <= 16;
+  const bool cl_ok = max_cpc_cl >= 1 && hp.nchunks <= 16 && W > T;
   // measured: the cluster pays while every CTA holds one chunk
   // (config 2: 1.50 vs 1.66 ms); with several chunks per CTA the staging of
   // 16 SMs loses to the grid's (config 3: 11.8 vs 10.7 ms)
@@ -612,14 +612,22 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
   // used runs win (config 4: 5.0 vs 10.8 us)
   hp.vec = trap_env("PM_TRAP_VEC", (int64_t)S * ldE * 4 <= (96ll << 20) ? 1 : 0);
-  const int32_t variant = trap_env("PM_TRAP_V", 0);
+  const int32_t variant = trap_env("PM_TRAP_V", -1);
   pm_status_t s;
   switch (variant) {
     case 1: s = launch_trap<1, 8>(hp, st); break;
     case 2: s = launch_trap<2, 8>(hp, st); break;
     case 3: s = launch_trap<4, 16>(hp, st); break;
     case 4: s = launch_trap<4, 8>(hp, st); break;
-    default: s = launch_trap<2, 16>(hp, st); break;
+    case 5: s = launch_trap<4, 32>(hp, st); break;
+    default:
+      // measured: 64-pair ranges x 16 classes while E is
+      // L2-resident; 128 x 32 from HBM while its 128-thread chunks fit one
+      // pass of the grid (config 4: 76.3 -> 67.9 ms; config 5 stays at
+      // 64 x 16: 1.21 vs 1.32 s)
+      if ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) s = launch_trap<4, 32>(hp, st);
+      else s = launch_trap<2, 16>(hp, st);
+      break;
   }
   if (s != PM_OK) return s;
   PM_CUDA_TRY(cudaFreeAsync(scratch, st));

@@ -531,7 +531,7 @@ def _check_trap(E_np):
 # ---- PM_LS_TRAP: every round on the temporal-blocked kernel (sparse hand-over
 # off), every compiled (pairs-per-lane, T) variant, chunk widths that do not
 # divide S/2, grid-barrier and cluster (DSMEM) modes.
-@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4, 5])
 @pytest.mark.parametrize("N,M,fam,W", [(128, 8, "smooth", 0), (512, 16, "smooth", 0), (512, 16, "ties", 7),
                                        (240, 8, "noise", 0), (336, 8, "smooth", 21), (128, 8, "transposition", 19)])
 @pytest.mark.parametrize("mode", ["0", "1"])
@@ -568,7 +568,7 @@ def test_local_search_padded_leading_dimension(method):
     assert (rounds, swaps) == (ref[1], ref[2])
 
 
-@pytest.mark.parametrize("variant,mode,vec", [("0", "0", "1"), ("0", "0", "0"), ("1", "1", "1"), ("3", "0", "1")])
+@pytest.mark.parametrize("variant,mode,vec", [("0", "0", "1"), ("0", "0", "0"), ("1", "1", "1"), ("3", "0", "1"), ("5", "0", "0")])
 def test_trap_every_round_config3(variant, mode, vec, monkeypatch):
     # S = 4096 with P = 768: pair-0 swaps at every u0 mod 4 (the 16-byte span offsets)
     monkeypatch.setenv("PM_TRAP_V", variant)
