@@ -64,7 +64,6 @@ struct TrapParams {
   LsResult* out;
   int64_t* per_round;
   int32_t* handoff;
-  unsigned long long* launches;
 };
 
 template <int PPL, int T>
@@ -303,7 +302,6 @@ k_ls_trap(const TrapParams p) {
   const int ngrp_tot = nblk * cpc;
   const int gid = blockIdx.x * cpc + grp;
 
-  if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p.launches, 1ull);
   if (p.out->status != PM_OK) return;   // grid-uniform (written before launch)
 
   if (threadIdx.x == 0) { s_cta_sw = 0; s_rsw[0] = s_rsw[1] = s_rsw[2] = 0ull; }
@@ -605,8 +603,6 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.sparse_T = sparse_T; hp.handoff = handoff;
   hp.bar = bar; hp.rsw = rsw;
   hp.out = dev_out; hp.per_round = dev_per_round;
-  hp.launches = device_launch_counter();
-  if (!hp.launches) return PM_ERR_CUDA;
   hp.prof = trap_env("PM_TRAP_PROF", 0);
   // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
