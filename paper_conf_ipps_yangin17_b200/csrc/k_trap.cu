@@ -52,8 +52,10 @@ namespace pm {
 struct TrapParams {
   const int32_t* E;
   int64_t ldE;
-  int32_t* rbuf[2];            // rbuf[0] = the caller's perm (grid mode: ping-pong)
-  int32_t* dbuf[2];
+  int32_t* rbuf[3];            // rbuf[0] = the caller's perm (grid mode: phase q reads q % 3)
+  int32_t* dbuf[3];
+  unsigned int* flags;         // grid mode, neighbour sync: phases completed per chunk
+  int32_t nbsync;              // grid mode: wait for the neighbour chunks only (W >= 2T)
   int32_t S, max_rounds, max_log, sparse_T;
   int32_t W, nchunks;
   int32_t gsz;                 // warps per chunk group (= PPL)
@@ -341,6 +343,7 @@ k_ls_trap(const TrapParams p) {
   unsigned long long t_ld = 0, t_st = 0, t_bar = 0, t_pub = 0, n_ph = 0, tq = prof ? gtimer() : 0;
   const int npass = (p.nchunks + ngrp_tot - 1) / ngrp_tot;
   uint32_t nph_cl = 0;   // cluster mode: phases completed (mbarrier parity)
+  uint32_t qph = 0;      // grid mode: phases completed
   for (;;) {
     if (!CLU && blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls; c0 += T) {
@@ -364,8 +367,26 @@ k_ls_trap(const TrapParams p) {
                                        [&](int32_t x, int32_t& g, int32_t& d) { const int2 v = rr[x]; g = v.x; d = v.y; },
                                        s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
           } else {
-            const int32_t* __restrict__ rc = cur ? p.rbuf[1] : p.rbuf[0];
-            const int32_t* __restrict__ dc = cur ? p.dbuf[1] : p.dbuf[0];
+            const int bi = p.nbsync ? (int)(qph % 3u) : cur;
+            const int32_t* __restrict__ rc = bi == 0 ? p.rbuf[0] : (bi == 1 ? p.rbuf[1] : p.rbuf[2]);
+            const int32_t* __restrict__ dc = bi == 0 ? p.dbuf[0] : (bi == 1 ? p.dbuf[1] : p.dbuf[2]);
+            if (p.nbsync && qph > 0) {
+              // the neighbour chunks' slots of phase qph - 1 (W >= 2T: every
+              // reader of this buffer's previous generation is within two
+              // chunks, and those finished it before our neighbours did theirs)
+              if (gt == 0) {
+#pragma unroll
+                for (int dch = -1; dch <= 1; dch += 2) {
+                  const int32_t c2 = ch + dch;
+                  if (c2 < 0 || c2 >= p.nchunks) continue;
+                  unsigned int v;
+                  do {
+                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.flags + c2) : "memory");
+                  } while (v < qph);
+                }
+              }
+              group_sync(1 + grp, GT);
+            }
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
                                        s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
@@ -395,8 +416,9 @@ k_ls_trap(const TrapParams p) {
                   st_async_v2(cluster_addr(a2, c2), g2, B.y, rm);
                 }
               } else {
-                int32_t* rn = cur ? p.rbuf[0] : p.rbuf[1];
-                int32_t* dn = cur ? p.dbuf[0] : p.dbuf[1];
+                const int bn = p.nbsync ? (int)((qph + 1u) % 3u) : (cur ^ 1);
+                int32_t* rn = bn == 0 ? p.rbuf[0] : (bn == 1 ? p.rbuf[1] : p.rbuf[2]);
+                int32_t* dn = bn == 0 ? p.dbuf[0] : (bn == 1 ? p.dbuf[1] : p.dbuf[2]);
                 __stcg(rn + x1, g1); __stcg(dn + x1, A.y);
                 __stcg(rn + x2, g2); __stcg(dn + x2, B.y);
               }
@@ -405,6 +427,10 @@ k_ls_trap(const TrapParams p) {
         }
         if (prof) { const unsigned long long t = gtimer(); t_pub += t - tq; }
         group_sync(1 + grp, GT);
+        if (!CLU && p.nbsync && have && gt == 0) {   // this chunk's slots of phase qph are out
+          __threadfence();
+          asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.flags + ch), "r"(qph + 1u) : "memory");
+        }
       }
       // swaps of this phase -> the round counter
 #pragma unroll
@@ -427,10 +453,11 @@ k_ls_trap(const TrapParams p) {
         mbar_wait_parity(&s_mbar[cur], (uint32_t)(nph_cl >> 1) & 1u);
         ++nph_cl;
         if (c0 + T >= ncls) cg::this_cluster().sync();   // round end: every CTA's s_rsw slot is set
-      } else {
+      } else if (!p.nbsync || c0 + T >= ncls) {   // neighbour sync: one grid barrier per round
         bar_target += nblk;
         grid_barrier(p.bar, bar_target);
       }
+      ++qph;
       if (prof) { const unsigned long long t = gtimer(); t_bar += t - tq; tq = t; ++n_ph; }
     }
     // round end (Alg. 2 lines 10-11)
@@ -478,9 +505,13 @@ k_ls_trap(const TrapParams p) {
       }
     }
     cg::this_cluster().sync();   // no CTA exits while others may still touch its smem
-  } else if (cur == 1) {   // the final state is in the scratch buffer: copy to perm
-    for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
-      p.rbuf[0][x] = __ldcg(p.rbuf[1] + x);
+  } else {   // the final state is in buffer qph % 3 (nbsync) or cur: copy to perm
+    const int bf = p.nbsync ? (int)(qph % 3u) : cur;
+    if (bf != 0) {
+      const int32_t* src = bf == 1 ? p.rbuf[1] : p.rbuf[2];
+      for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
+        p.rbuf[0][x] = __ldcg(src + x);
+    }
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     p.out->status = status;
@@ -556,7 +587,9 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
     note_launch();
     return PM_OK;
   }
-  // grid mode: cpc chunk groups per CTA, enough CTAs for one pass if possible
+  // grid mode: cpc chunk groups per CTA, enough CTAs for one pass if possible;
+  // neighbour synchronisation (chunk flags, three state buffers) when W >= 2T
+  hp.nbsync = (W >= 2 * T) ? trap_env("PM_TRAP_NBSYNC", 1) : 0;
   int max_cpc = (int)((size_t)optin / SM::bytes);
   if (max_cpc > 8 / gsz) max_cpc = 8 / gsz;
   if (max_cpc < 1) return PM_ERR_UNSUPPORTED;
@@ -586,19 +619,23 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
                      int32_t* handoff, int32_t sparse_T) {
   if (S < ls_trap_min_S() || (S & 1)) return PM_ERR_UNSUPPORTED;
   PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
-  // scratch: r1 [S], d0 [S], d1 [S], barrier counter, 3 round counters
+  // scratch: 3 round counters, barrier counter, chunk flags [S/2], r1, r2,
+  // d0, d1, d2 [S]
   const size_t n = (size_t)S;
   char* scratch = nullptr;
-  const size_t bytes = sizeof(int32_t) * 3 * n + 64 + sizeof(unsigned long long) * 3;
+  const size_t head = 64 + sizeof(unsigned int) * (n / 2 + 16);
+  const size_t bytes = head + sizeof(int32_t) * 5 * n;
   PM_CUDA_TRY(pm::scratch_alloc(reinterpret_cast<void**>(&scratch), bytes, st));
   unsigned long long* rsw = reinterpret_cast<unsigned long long*>(scratch);
   unsigned int* bar = reinterpret_cast<unsigned int*>(scratch + 32);
-  int32_t* base = reinterpret_cast<int32_t*>(scratch + 64);
-  PM_CUDA_TRY(cudaMemsetAsync(scratch, 0, 64, st));
+  unsigned int* flags = reinterpret_cast<unsigned int*>(scratch + 64);
+  int32_t* base = reinterpret_cast<int32_t*>(scratch + head);
+  PM_CUDA_TRY(cudaMemsetAsync(scratch, 0, head, st));
   TrapParams hp = {};
   hp.E = E; hp.ldE = ldE;
-  hp.rbuf[0] = perm; hp.rbuf[1] = base;
-  hp.dbuf[0] = base + n; hp.dbuf[1] = base + 2 * n;
+  hp.rbuf[0] = perm; hp.rbuf[1] = base; hp.rbuf[2] = base + n;
+  hp.dbuf[0] = base + 2 * n; hp.dbuf[1] = base + 3 * n; hp.dbuf[2] = base + 4 * n;
+  hp.flags = flags;
   hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
   hp.sparse_T = sparse_T; hp.handoff = handoff;
   hp.bar = bar; hp.rsw = rsw;
