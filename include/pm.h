@@ -24,6 +24,7 @@
 #ifndef PM_H_
 #define PM_H_
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -163,6 +164,40 @@ pm_status_t pm_local_search_ex(const int32_t* d_E, int64_t ld_E, int32_t S, int3
 pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
                                   int32_t max_rounds, int32_t method, int64_t* d_result,
                                   pm_stream_t stream);
+
+/* Multi-GPU Algorithm 2 (method PM_LS_TRAP split across ranks,
+ * one rank per GPU of one NVLink box).  The colour classes are global
+ * perfect matchings, so the search does not shard into independent parts;
+ * instead rank r runs the TRAP phases on its contiguous share of the pair
+ * chunks and exchanges, per phase, only the slots of the chunks at its range
+ * ends with its neighbour ranks -- peer stores of (r, d) plus a phase flag
+ * (release/acquire at system scope) into their workspaces -- and, once per
+ * round, the round's swap count (peer atomics + a cross-rank barrier).
+ * Every rank holds the whole of E (replicated; e.g. gathered from the
+ * row shards of pm_error_matrix).  Results are bit-identical to
+ * pm_local_search.
+ *   pm_trap_workspace_bytes : per-rank workspace size for S.
+ *   pm_trap_workspace_reset : zero a workspace's counters and flags (every
+ *            rank's, followed by a cross-process barrier, before a search).
+ *   pm_local_search_multi_async : this rank's part; d_perm_peers[o] and
+ *            d_ws_peers[o] (host arrays of `world` device pointers) are rank
+ *            o's perm (int32 [S], the same bijection on every rank on entry,
+ *            the final r on every rank on exit) and workspace, mapped into
+ *            this process (peer access / IPC); d_result as
+ *            pm_local_search_async (this rank's copy).  All ranks must run
+ *            concurrently (the kernels wait on each other).
+ *   pm_local_search_multi_emulated : test hook -- all `world` ranks in one
+ *            launch on the current device (own workspaces and perms), the
+ *            exchange protocol unchanged; d_perm in/out as pm_local_search.
+ * world <= 8; S even, >= 256, and S/64 >= world. */
+size_t pm_trap_workspace_bytes(int32_t S);
+pm_status_t pm_trap_workspace_reset(void* d_ws, int32_t S, pm_stream_t stream);
+pm_status_t pm_local_search_multi_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* const* d_perm_peers,
+                                        void* const* d_ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
+                                        int64_t* d_result, pm_stream_t stream);
+pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                           int32_t world, int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
+                                           pm_stream_t stream);
 
 /* The method PM_LS_AUTO selects for S on the current device (host-only). */
 int32_t pm_ls_auto_method(int32_t S);

@@ -667,4 +667,326 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   return PM_OK;
 }
 
+
+// =====================================================================
+// Multi-rank TRAP (one rank per GPU; NVLink peer memory).  The chunks are
+// split into `world` contiguous ranges; rank r runs the grid-mode phases on
+// its range with the neighbour synchronisation above, except that a chunk
+// publishes its owned slots (and its phase flag) to the rank(s) owning
+// chunks ch-1, ch, ch+1 -- by peer stores when another rank owns them.  E
+// is replicated (every rank holds all of it).  Once per round every rank
+// adds its swap count to every rank's round total and passes a cross-rank
+// barrier; at the end every chunk writes its owned slots' final tiles into
+// every rank's perm, so every rank returns the whole result.  The same
+// kernel runs all ranks inside one launch on one device for the test hook
+// pm_local_search_multi_emulated (peer pointers are then plain pointers).
+constexpr int kMaxRanks = 8;
+struct TrapRank {                 // one rank's workspace (see trap_ws_layout)
+  int32_t* rbuf[3];
+  int32_t* dbuf[3];
+  unsigned int* flags;            // [nchunks] phases completed, per chunk
+  unsigned int* bar;              // this rank's grid barrier counter
+  unsigned int* xbar;             // cross-rank barrier counter
+  unsigned long long* rtot;       // [3] round swap totals (all ranks add)
+  int32_t* perm;
+  const int32_t* E;
+};
+struct TrapMultiParams {
+  TrapRank rk[kMaxRanks];
+  int64_t ldE;
+  int32_t S, max_rounds, max_log, W, nchunks, world, rank0, ctas_per_rank, vec;
+  LsResult* out;                  // written by the launch's first rank
+  int64_t* per_round;
+};
+
+__device__ __forceinline__ int32_t chunk_begin(int32_t r, int32_t nchunks, int32_t world) {
+  return (int32_t)(((int64_t)r * nchunks) / world);
+}
+__device__ __forceinline__ int32_t chunk_owner(int32_t ch, int32_t nchunks, int32_t world) {
+  int32_t r = 0;
+  while (r + 1 < world && chunk_begin(r + 1, nchunks, world) <= ch) ++r;
+  return r;
+}
+__device__ __forceinline__ void sys_barrier_arrive_wait(const TrapMultiParams& p, int32_t r, unsigned int target) {
+  // every rank's leader: arrive at every rank's counter, wait for its own
+  __threadfence_system();
+  for (int o = 0; o < p.world; ++o)
+    asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(p.rk[o].xbar) : "memory");
+  unsigned int v;
+  do {
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p.rk[r].xbar) : "memory");
+  } while (v < target);
+}
+
+template <int PPL, int T>
+__global__ void __launch_bounds__(256, 1)
+k_ls_trap_mr(const TrapMultiParams p) {
+  using SM = TrapSmem<PPL, T>;
+  constexpr int L = SM::L, X = SM::X, GT = X;
+  extern __shared__ __align__(16) int32_t sm[];
+  const int cpc = blockDim.x / GT;
+  const int grp = threadIdx.x / GT;
+  const int gt = threadIdx.x - grp * GT;
+  int32_t* ws = sm + (size_t)grp * SM::ints;
+  int4* s_st = reinterpret_cast<int4*>(ws);
+  int32_t* s_g = ws + 4 * L;
+  int32_t* s_E = s_g + L;
+  __shared__ int32_t s_cta_sw;
+  __shared__ unsigned long long s_rs;
+
+  const int32_t r = p.rank0 + (int32_t)(blockIdx.x / p.ctas_per_rank);
+  const int32_t lb = (int32_t)(blockIdx.x % p.ctas_per_rank);
+  const bool leader = (lb == 0 && threadIdx.x == 0);
+  const TrapRank& me = p.rk[r];
+  const int32_t* __restrict__ E = me.E;
+  const int64_t ld = p.ldE;
+  const int32_t S = p.S;
+  const bool vec = p.vec && ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);
+  const Classes cl(S);
+  const int32_t m = cl.m, H = cl.half, K = cl.npairs - 1, ncls = cl.ncls;
+  const int32_t W = p.W, world = p.world, nch = p.nchunks;
+  const int32_t cb = chunk_begin(r, nch, world), ce = chunk_begin(r + 1, nch, world);
+  const unsigned nloc = p.ctas_per_rank;
+  unsigned int bar_target = 0;
+  if (p.out->status != PM_OK) return;   // uniform (written before launch)
+
+  if (threadIdx.x == 0) s_cta_sw = 0;
+  for (int32_t x = lb * blockDim.x + threadIdx.x; x < S; x += nloc * blockDim.x)
+    __stcg(me.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(me.rbuf[0] + x) * ld + x));
+  bar_target += nloc;
+  grid_barrier(me.bar, bar_target);
+
+  uint32_t q = 0;
+  int32_t rounds = 0;
+  int64_t total = 0;
+  int status = PM_OK;
+  unsigned int xtarget = 0;
+  for (;;) {
+    if (leader) me.rtot[(rounds + 1) % 3] = 0ull;
+    for (int32_t c0 = 0; c0 < ncls; c0 += T) {
+      const int32_t Tp = min(T, ncls - c0);
+      const int32_t u0 = wrap_m(c0 + H, m);
+      const int bi = (int)(q % 3u), bn = (int)((q + 1u) % 3u);
+      int mysw = 0;
+      for (int32_t ch = cb + lb * cpc + grp; ch < ce + (int32_t)(nloc * cpc); ch += (int32_t)(nloc * cpc)) {
+        const bool have = ch < ce;
+        if (have && q > 0 && gt == 0) {
+          for (int dch = -1; dch <= 1; dch += 2) {
+            const int32_t c2 = ch + dch;
+            if (c2 < 0 || c2 >= nch) continue;
+            unsigned int v;
+            do {
+              asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(me.flags + c2) : "memory");
+            } while (v < q);
+          }
+        }
+        group_sync(1 + grp, GT);
+        if (have) {
+          TrapChunk C;
+          const int32_t k0 = ch * W, k1 = min(k0 + W, K + 1);
+          C.a = max(k0 - Tp, 0); C.b = min(k1 + Tp, K + 1);
+          C.a2 = max(C.a, 1);
+          C.nA = C.b - C.a; C.nB = C.b - C.a2;
+          C.Lc = C.nA + C.nB + (C.a == 0 ? 1 : 0);
+          C.K = K; C.m = m; C.Tp = Tp;
+          const int32_t* __restrict__ rc = me.rbuf[bi];
+          const int32_t* __restrict__ dc = me.dbuf[bi];
+          mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
+                                     [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
+                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr);
+          // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
+          int32_t own[3];
+          int nown = 0;
+          for (int dch = -1; dch <= 1; ++dch) {
+            const int32_t c2 = ch + dch;
+            if (c2 < 0 || c2 >= nch) continue;
+            const int32_t o = chunk_owner(c2, nch, world);
+            bool dup = false;
+            for (int i = 0; i < nown; ++i) dup |= (own[i] == o);
+            if (!dup) own[nown++] = o;
+          }
+          const int32_t k = C.a + gt;
+          if (k >= k0 && k < k1) {
+            int32_t j1, j2;
+            C.local_slots(Tp - 1, k, j1, j2);
+            const int32_t x1 = C.slot_of(j1, u0, S), x2 = C.slot_of(j2, u0, S);
+            const int4 A = s_st[j1], B = s_st[j2];
+            const int32_t g1 = s_g[A.x & 0xffff], g2 = s_g[B.x & 0xffff];
+            for (int i = 0; i < nown; ++i) {
+              const TrapRank& ro = p.rk[own[i]];
+              __stcg(ro.rbuf[bn] + x1, g1); __stcg(ro.dbuf[bn] + x1, A.y);
+              __stcg(ro.rbuf[bn] + x2, g2); __stcg(ro.dbuf[bn] + x2, B.y);
+            }
+          }
+          group_sync(1 + grp, GT);
+          if (gt == 0) {
+            __threadfence_system();
+            for (int i = 0; i < nown; ++i)
+              asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p.rk[own[i]].flags + ch), "r"(q + 1u)
+                           : "memory");
+          }
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) mysw += __shfl_xor_sync(0xffffffffu, mysw, o);
+      if ((threadIdx.x & 31) == 0 && mysw) atomicAdd(&s_cta_sw, mysw);
+      ++q;
+      __syncthreads();
+      if (c0 + T >= ncls) {
+        // round end: every CTA's count to every rank's total, then the rank
+        // barrier and the cross-rank barrier, then the rank barrier again
+        if (threadIdx.x == 0 && s_cta_sw) {
+          for (int o = 0; o < world; ++o) atomicAdd(p.rk[o].rtot + rounds % 3, (unsigned long long)s_cta_sw);
+        }
+        if (threadIdx.x == 0) s_cta_sw = 0;
+        bar_target += nloc;
+        grid_barrier(me.bar, bar_target);
+        if (leader) {
+          xtarget += (unsigned)world;
+          sys_barrier_arrive_wait(p, r, xtarget);
+        }
+        bar_target += nloc;
+        grid_barrier(me.bar, bar_target);
+      }
+    }
+    if (threadIdx.x == 0) s_rs = *((volatile unsigned long long*)(me.rtot + rounds % 3));
+    __syncthreads();
+    const int64_t rs = (int64_t)s_rs;
+    if (leader && r == p.rank0 && rounds < p.max_log) p.per_round[rounds] = rs;
+    rounds += 1;
+    total += rs;
+    __syncthreads();
+    if (rs == 0) break;
+    if (p.max_rounds > 0 && rounds >= p.max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
+  }
+  // every chunk's owned slots (class ncls - 1) into every rank's perm
+  const int32_t* fin = me.rbuf[q % 3u];
+  for (int32_t ch = cb + lb * cpc + grp; ch < ce; ch += (int32_t)(nloc * cpc)) {
+    const int32_t k0 = ch * W, k1 = min(k0 + W, K + 1);
+    for (int32_t k = k0 + gt; k < k1; k += GT) {
+      int32_t u, v;
+      cl.pair(ncls - 1, k, u, v);
+      const int32_t gu = __ldcg(fin + u), gv = __ldcg(fin + v);
+      for (int o = 0; o < world; ++o) {
+        __stcg(p.rk[o].perm + u, gu);
+        __stcg(p.rk[o].perm + v, gv);
+      }
+    }
+  }
+  bar_target += nloc;
+  grid_barrier(me.bar, bar_target);
+  if (leader) {
+    xtarget += (unsigned)world;
+    sys_barrier_arrive_wait(p, r, xtarget);
+    if (r == p.rank0) {
+      p.out->status = status;
+      p.out->rounds = rounds;
+      p.out->swaps = total;
+    }
+  }
+}
+
+// Per-rank workspace: 3 round totals, barrier counters, chunk flags, r1, r2,
+// d0, d1, d2 (the rank's perm is r0).
+size_t trap_ws_bytes(int32_t S) {
+  const size_t n = (size_t)S;
+  return 128 + sizeof(unsigned int) * (n / 2 + 16) + sizeof(int32_t) * 5 * n;
+}
+static void trap_ws_layout(void* ws, int32_t S, int32_t* perm, const int32_t* E, TrapRank& rk) {
+  const size_t n = (size_t)S;
+  char* b = static_cast<char*>(ws);
+  rk.rtot = reinterpret_cast<unsigned long long*>(b);
+  rk.bar = reinterpret_cast<unsigned int*>(b + 32);
+  rk.xbar = reinterpret_cast<unsigned int*>(b + 64);
+  rk.flags = reinterpret_cast<unsigned int*>(b + 128);
+  int32_t* base = reinterpret_cast<int32_t*>(b + 128 + sizeof(unsigned int) * (n / 2 + 16));
+  rk.rbuf[0] = perm; rk.rbuf[1] = base; rk.rbuf[2] = base + n;
+  rk.dbuf[0] = base + 2 * n; rk.dbuf[1] = base + 3 * n; rk.dbuf[2] = base + 4 * n;
+  rk.perm = perm;
+  rk.E = E;
+}
+size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((size_t)S / 2 + 16); }
+
+// Launch `nloc` ranks [rank0, rank0 + nloc) of a world on the current device.
+pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
+                           int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
+                           cudaStream_t st) {
+  constexpr int PPL = 2, T = 16;
+  using SM = TrapSmem<PPL, T>;
+  if (S < ls_trap_min_S() || (S & 1) || world < 1 || world > kMaxRanks || nloc < 1) return PM_ERR_UNSUPPORTED;
+  int dev = 0, nsm = 0, optin = 0;
+  PM_CUDA_TRY(cudaGetDevice(&dev));
+  PM_CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  PM_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  TrapMultiParams hp = {};
+  for (int i = 0; i < world; ++i) hp.rk[i] = ranks[i];
+  hp.ldE = ldE; hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
+  hp.W = SM::X - 2 * T;    // W = 2T: the neighbour synchronisation holds
+  hp.nchunks = (Classes(S).npairs + hp.W - 1) / hp.W;
+  if (hp.nchunks < world) return PM_ERR_UNSUPPORTED;
+  hp.world = world; hp.rank0 = rank0;
+  hp.vec = ((int64_t)S * ldE * 4 <= (96ll << 20)) ? 1 : 0;
+  hp.out = dev_out; hp.per_round = dev_per_round;
+  const int per_rank_chunks = (hp.nchunks + world - 1) / world;
+  int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
+  int max_cpc = (int)((size_t)optin / SM::bytes);
+  if (max_cpc > 8 / PPL) max_cpc = 8 / PPL;
+  if (cpc < 1) cpc = 1;
+  if (cpc > max_cpc) cpc = max_cpc;
+  const size_t smem = SM::bytes * cpc;
+  const int threads = SM::X * cpc;
+  auto fn = k_ls_trap_mr<PPL, T>;
+  PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int occ = 0;
+  PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
+  if (occ < 1) return PM_ERR_UNSUPPORTED;
+  int cpr = (per_rank_chunks + cpc - 1) / cpc;        // CTAs per rank
+  if (cpr * nloc > nsm * occ) cpr = (nsm * occ) / nloc;
+  if (cpr < 1) return PM_ERR_UNSUPPORTED;
+  hp.ctas_per_rank = cpr;
+  void* args[] = {(void*)&hp};
+  PM_CUDA_TRY(cudaLaunchCooperativeKernel((const void*)fn, dim3(cpr * nloc), dim3(threads), args, smem, st));
+  note_launch();
+  return PM_OK;
+}
+
+
+// All ranks of a world on the current device, one launch (test hook).
+pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
+                                int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
+                                cudaStream_t st) {
+  if (world < 1 || world > kMaxRanks) return PM_ERR_UNSUPPORTED;
+  PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
+  const size_t wsb = (trap_ws_bytes(S) + 255) / 256 * 256;
+  const size_t pb = ((size_t)S * sizeof(int32_t) + 255) / 256 * 256;
+  char* buf = nullptr;
+  PM_CUDA_TRY(pm::scratch_alloc(reinterpret_cast<void**>(&buf), (wsb + pb) * world, st));
+  TrapRank ranks[kMaxRanks];
+  for (int r = 0; r < world; ++r) {
+    char* ws = buf + (wsb + pb) * r;
+    int32_t* pr = reinterpret_cast<int32_t*>(ws + wsb);
+    PM_CUDA_TRY(cudaMemsetAsync(ws, 0, trap_ws_zero_bytes(S), st));
+    PM_CUDA_TRY(cudaMemcpyAsync(pr, perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
+    trap_ws_layout(ws, S, pr, E, ranks[r]);
+  }
+  pm_status_t s = run_trap_multi(ranks, world, 0, world, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st);
+  if (s != PM_OK) return s;
+  // every rank holds the whole result; return rank world-1's (the farthest)
+  PM_CUDA_TRY(cudaMemcpyAsync(perm, ranks[world - 1].perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
+  PM_CUDA_TRY(cudaFreeAsync(buf, st));
+  return PM_OK;
+}
+
+// One rank of a multi-GPU world: ws_peers[o] / perm_peers[o] are rank o's
+// workspace and perm mapped into this process (peer memory); every
+// workspace zeroed and every perm holding the same bijection before any
+// rank launches.
+pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* const* perm_peers,
+                            void* const* ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
+                            LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
+  if (world < 1 || world > kMaxRanks || rank < 0 || rank >= world) return PM_ERR_INVALID;
+  TrapRank ranks[kMaxRanks];
+  for (int r = 0; r < world; ++r) trap_ws_layout(ws_peers[r], S, perm_peers[r], E, ranks[r]);
+  return run_trap_multi(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st);
+}
 }  // namespace pm

@@ -249,6 +249,47 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
                           nullptr, 0, st, &used);
 }
 
+size_t pm_trap_workspace_bytes(int32_t S) { return (S < 2) ? 0 : trap_ws_bytes(S); }
+
+pm_status_t pm_trap_workspace_reset(void* d_ws, int32_t S, pm_stream_t stream) {
+  if (!d_ws || S < 2) return PM_ERR_INVALID;
+  PM_CUDA_TRY(cudaMemsetAsync(d_ws, 0, trap_ws_zero_bytes(S), (cudaStream_t)stream));
+  return PM_OK;
+}
+
+pm_status_t pm_local_search_multi_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* const* d_perm_peers,
+                                        void* const* d_ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
+                                        int64_t* d_result, pm_stream_t stream) {
+  if (!d_E || !d_perm_peers || !d_ws_peers || !d_result || ld_E < S || max_rounds < 0) return PM_ERR_INVALID;
+  if (world < 1 || rank < 0 || rank >= world) return PM_ERR_INVALID;
+  for (int r = 0; r < world; ++r)
+    if (!d_perm_peers[r] || !d_ws_peers[r]) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
+  return trap_multi_rank(d_E, ld_E, S, d_perm_peers, d_ws_peers, rank, world, max_rounds,
+                         reinterpret_cast<LsResult*>(d_result), nullptr, 0, st);
+}
+
+pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                           int32_t world, int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
+                                           pm_stream_t stream) {
+  if (!d_E || !d_perm || ld_E < S || max_rounds < 0 || world < 1) return PM_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  DevBuf buf;
+  buf.st = st;
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, sizeof(LsResult), st));
+  LsResult* dres = reinterpret_cast<LsResult*>(buf.p);
+  PM_CUDA_TRY(cudaMemsetAsync(dres, 0, sizeof(LsResult), st));
+  pm_status_t s = trap_multi_emulated(d_E, ld_E, S, d_perm, world, max_rounds, dres, nullptr, 0, st);
+  if (s != PM_OK) return s;
+  LsResult h;
+  PM_CUDA_TRY(cudaMemcpyAsync(&h, dres, sizeof(h), cudaMemcpyDeviceToHost, st));
+  PM_CUDA_TRY(cudaStreamSynchronize(st));
+  if (h_rounds) *h_rounds = (int32_t)h.rounds;
+  if (h_swaps) *h_swaps = h.swaps;
+  return (pm_status_t)h.status;
+}
+
 int32_t pm_ls_cta_max_S(void) { return ls_cta_max_S(); }
 
 int32_t pm_ls_auto_method(int32_t S) {

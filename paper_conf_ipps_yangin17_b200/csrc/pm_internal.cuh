@@ -173,6 +173,17 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
                      LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
                      int32_t* handoff, int32_t sparse_T);
 
+// Multi-rank TRAP (k_trap.cu).
+struct TrapRank;
+size_t trap_ws_bytes(int32_t S);
+size_t trap_ws_zero_bytes(int32_t S);
+pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
+                                int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
+                                cudaStream_t st);
+pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* const* perm_peers,
+                            void* const* ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
+                            LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
+
 // Exact min-weight perfect matching by eps-scaling auction (k_assign.cu).
 // h_stats (nullable): {bidding rounds, phases}.  Synchronises st.
 pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* perm, int64_t* price_out,

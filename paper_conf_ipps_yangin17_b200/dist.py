@@ -74,3 +74,40 @@ def sum_over_ranks(value: float, device=None, group=None) -> float:
     t = torch.tensor([float(value)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     return float(t.item())
+
+
+def local_search_multi(E: torch.Tensor, perm: torch.Tensor | None = None, max_rounds: int = 0, group=None):
+    """Algorithm 2 across the ranks of `group` (one per GPU of one NVLink box)
+    with pm_local_search_multi_async: every rank passes the full E
+    (replicated, e.g. from error_matrix_sharded(..., gather=True)) and the
+    same initial perm; every rank returns the final r.  The per-rank
+    workspaces and perms live in torch symmetric memory, so each rank sees
+    the others' as peer pointers.  Returns (perm, rounds, swaps)."""
+    import torch.distributed._symmetric_memory as symm_mem
+
+    from . import pm
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    S = E.shape[0]
+    ws_bytes = (pm.trap_workspace_bytes(S) + 255) // 256 * 256
+    buf = symm_mem.empty(ws_bytes + 4 * S, dtype=torch.uint8, device=E.device)
+    name = (group or dist.group.WORLD).group_name
+    hdl = symm_mem.rendezvous(buf, name)
+    ptrs = [int(p) for p in hdl.buffer_ptrs]
+    my_perm = buf[ws_bytes:].view(torch.int32)
+    my_perm.copy_(torch.arange(S, dtype=torch.int32, device=E.device) if perm is None else perm)
+    buf[:ws_bytes].zero_()
+    torch.cuda.synchronize(E.device)
+    dist.barrier(group)                                   # every workspace reset before any rank starts
+    result = torch.zeros(3, dtype=torch.int64, device=E.device)
+    pm.local_search_multi_async(E, [p + ws_bytes for p in ptrs], ptrs, rank, world, result, max_rounds=max_rounds)
+    torch.cuda.synchronize(E.device)
+    dist.barrier(group)                                   # no rank frees its buffer while peers may write it
+    status, rounds, swaps = (int(v) for v in result.tolist())
+    if status not in (0, 3):
+        raise pm.PMError(status, "pm_local_search_multi_async")
+    out = my_perm.clone()
+    if perm is not None:
+        perm.copy_(out)
+        out = perm
+    return out, rounds, swaps

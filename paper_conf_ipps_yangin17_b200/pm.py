@@ -49,6 +49,10 @@ _SIGS = [
     ("pm_render", ctypes.c_int, [_P, _I32, _I32, _I32, _P, _P, _P]),
     ("pm_optimal_assignment", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P, _P, _P]),
     ("pm_launch_count", _I64, []),
+    ("pm_trap_workspace_bytes", ctypes.c_size_t, [_I32]),
+    ("pm_trap_workspace_reset", ctypes.c_int, [_P, _I32, _P]),
+    ("pm_local_search_multi_async", ctypes.c_int, [_P, _I64, _I32, _P, _P, _I32, _I32, _I32, _P, _P]),
+    ("pm_local_search_multi_emulated", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P]),
 ]
 
 
@@ -206,6 +210,36 @@ def local_search_async(E, perm, result, max_rounds: int = 0, method: str = "auto
     _check(lib().pm_local_search_async(E.data_ptr(), E.stride(0), E.shape[0], perm.data_ptr(), max_rounds,
                                        METHODS[method], result.data_ptr(), _stream(stream)),
            "pm_local_search_async")
+
+
+def local_search_multi_emulated(E, world: int, perm=None, max_rounds: int = 0, stream=None):
+    """pm_local_search_multi_emulated (test hook): the multi-GPU TRAP protocol
+    with `world` ranks in one launch on this device.  Returns (perm, rounds, swaps)."""
+    torch = _torch()
+    _dev(E, torch.int32)
+    S = E.shape[0]
+    if perm is None:
+        perm = torch.arange(S, dtype=torch.int32, device=E.device)
+    rounds, swaps = ctypes.c_int32(0), ctypes.c_int64(0)
+    _check(lib().pm_local_search_multi_emulated(E.data_ptr(), E.stride(0), S, perm.data_ptr(), world, max_rounds,
+                                                ctypes.byref(rounds), ctypes.byref(swaps), _stream(stream)),
+           "pm_local_search_multi_emulated", (PM_OK, PM_ERR_NOT_CONVERGED))
+    return perm, int(rounds.value), int(swaps.value)
+
+
+def trap_workspace_bytes(S: int) -> int:
+    return int(lib().pm_trap_workspace_bytes(S))
+
+
+def local_search_multi_async(E, perm_ptrs, ws_ptrs, rank: int, world: int, result, max_rounds: int = 0,
+                             stream=None):
+    """pm_local_search_multi_async: this rank's part of the multi-GPU search;
+    perm_ptrs / ws_ptrs = every rank's perm / workspace device pointers as
+    mapped into this process (ints)."""
+    P = ctypes.c_void_p * world
+    _check(lib().pm_local_search_multi_async(E.data_ptr(), E.stride(0), E.shape[0], P(*perm_ptrs), P(*ws_ptrs),
+                                             rank, world, max_rounds, result.data_ptr(), _stream(stream)),
+           "pm_local_search_multi_async")
 
 
 def ls_cta_max_S() -> int:

@@ -576,3 +576,51 @@ def test_trap_every_round_config3(variant, mode, vec, monkeypatch):
     monkeypatch.setenv("PM_TRAP_VEC", vec)
     monkeypatch.setenv("PM_LS_SPARSE", "0")
     _check_trap(oracle_E("smooth", 1024, 16))
+
+
+# ---- multi-GPU TRAP protocol (pm_local_search_multi_*): every rank of a world
+# emulated in one launch on this GPU -- chunk ranges per rank, halo slots and
+# phase flags to the neighbour ranks' workspaces, per-round cross-rank swap
+# totals and barrier, the final r on every rank -- against the oracle.
+@pytest.mark.parametrize("N,M,fam,world", [(128, 8, "smooth", 2), (128, 8, "noise", 4), (512, 16, "smooth", 1),
+                                           (512, 16, "smooth", 2), (512, 16, "ties", 3), (512, 16, "smooth", 8),
+                                           (1024, 16, "smooth", 4), (336, 8, "transposition", 5)])
+def test_multi_rank_trap_emulated(N, M, fam, world):
+    E_np = oracle_E(fam, N, M)
+    ref = oracle.local_search(E_np)
+    out, rounds, swaps = pm.local_search_multi_emulated(dev(E_np), world)
+    assert (out.cpu().numpy() == ref[0]).all()
+    assert (rounds, swaps) == (ref[1], ref[2])
+
+
+def test_multi_rank_trap_max_rounds_then_resume():
+    E_np = oracle_E("smooth", 512, 16)
+    ref = oracle.local_search(E_np, max_rounds=2)
+    out, rounds, swaps = pm.local_search_multi_emulated(dev(E_np), 3, max_rounds=2)
+    assert (out.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    ref2 = oracle.local_search(E_np, r0=ref[0])
+    out2, rounds2, swaps2 = pm.local_search_multi_emulated(dev(E_np), 3, perm=out)
+    assert (out2.cpu().numpy() == ref2[0]).all() and (rounds2, swaps2) == (ref2[1], ref2[2])
+
+
+def test_multi_rank_trap_symmetric_memory_world1():
+    # the multi-process plumbing (torch symmetric memory, peer pointer table,
+    # workspace reset + barrier) through pm_local_search_multi_async, at one rank
+    import torch.distributed as tdist
+
+    from paper_conf_ipps_yangin17_b200 import dist as pdist
+    E_np = oracle_E("smooth", 512, 16)
+    ref = oracle.local_search(E_np)
+    own = not tdist.is_initialized()
+    if own:
+        tdist.init_process_group("nccl", init_method="tcp://127.0.0.1:29513", rank=0, world_size=1,
+                                 device_id=torch.device(DEV))
+    try:
+        try:
+            out, rounds, swaps = pdist.local_search_multi(dev(E_np))
+        except (RuntimeError, AttributeError) as e:
+            pytest.skip(f"symmetric memory unavailable here: {e}")
+        assert (out.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    finally:
+        if own:
+            tdist.destroy_process_group()
