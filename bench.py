@@ -53,6 +53,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="budget of the cpu_baseline sample")
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--sharded", action="store_true",
+                    help="one photomosaic for the whole job (strong scaling): E row-sharded + all-gathered "
+                         "(NCCL), Alg. 2 across the ranks (pm_local_search_multi_async over symmetric memory)")
     return ap.parse_args()
 
 
@@ -319,6 +322,95 @@ def bench_ours(args, rank, world, local_rank):
     return line, (I_np, T_np, M, S, perm.cpu().numpy(), out_res)
 
 
+
+def bench_sharded(args, rank, world, local_rank):
+    """One photomosaic for the whole job: every rank computes its row shard of
+    E (pm_error_matrix rows), NCCL all-gathers E, and Algorithm 2 runs across
+    the ranks (pm_local_search_multi_async: per-rank chunk ranges, halo slots
+    by NVLink peer stores).  value = S^2 / step time (strong scaling)."""
+    import torch
+    import torch.distributed as dist
+    import torch.distributed._symmetric_memory as symm_mem
+
+    from paper_conf_ipps_yangin17_b200 import dist as pdist
+    from paper_conf_ipps_yangin17_b200 import pm, synth
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world == 1 and not dist.is_initialized():
+        dist.init_process_group("nccl", init_method="tcp://127.0.0.1:29517", rank=0, world_size=1, device_id=dev)
+    cfg = synth.CONFIGS[args.config]
+    N, M, C = cfg["N"], cfg["M"], cfg["C"]
+    S = (N // M) ** 2
+    I_np, T_np = synth.make_pair(args.family, N, M, C, seed=0)       # the same photomosaic on every rank
+    dI = torch.from_numpy(I_np).to(dev)
+    dT = torch.from_numpy(T_np).to(dev)
+    b, e = pdist.shard_rows(S, world, rank)
+    rows_max = max(pdist.shard_rows(S, world, g)[1] - pdist.shard_rows(S, world, g)[0] for g in range(world))
+    parts = torch.zeros((world, rows_max, S), dtype=torch.int32, device=dev)
+    part = parts[rank]                                                   # in-place all-gather
+    sizes = [pdist.shard_rows(S, world, g) for g in range(world)]
+    contiguous = all(se - sb == rows_max for sb, se in sizes)
+    E_full = parts.view(world * rows_max, S) if contiguous else torch.empty((S, S), dtype=torch.int32, device=dev)
+    ws_bytes = (pm.trap_workspace_bytes(S) + 255) // 256 * 256
+    buf = symm_mem.empty(ws_bytes + 4 * S, dtype=torch.uint8, device=dev)
+    hdl = symm_mem.rendezvous(buf, dist.group.WORLD.group_name)
+    ptrs = [int(p) for p in hdl.buffer_ptrs]
+    my_perm = buf[ws_bytes:].view(torch.int32)
+    res = torch.zeros(3, dtype=torch.int64, device=dev)
+    cost = torch.zeros(1, dtype=torch.int64, device=dev)
+    token = torch.zeros(1, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(evs=None):
+        if evs: evs[0].record(stream)
+        pm.error_matrix(dI, dT, M, rows=(b, e), out=part[: e - b])        # Step 1+2, this rank's rows
+        if evs: evs[1].record(stream)
+        if world > 1:
+            dist.all_gather_into_tensor(parts.view(world * rows_max, S), part)
+            if not contiguous:
+                for g, (sb, se) in enumerate(sizes):
+                    E_full[sb:se].copy_(parts[g, : se - sb])
+        if evs: evs[2].record(stream)
+        pm.init_identity(my_perm)
+        pm.trap_workspace_reset(buf, S)
+        dist.all_reduce(token)                                             # every workspace reset (device order)
+        pm.local_search_multi_async(E_full, [p + ws_bytes for p in ptrs], ptrs, rank, world, res)
+        if evs: evs[3].record(stream)
+        pm.cost_async(E_full, my_perm, cost)
+        if evs: evs[4].record(stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    ref = res.cpu().tolist() + cost.cpu().tolist()
+    K = args.steps
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(K)]
+    dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local_rank) as clk:
+        for i in range(K):
+            step(evs[i])
+        torch.cuda.synchronize()
+    dist.barrier()
+    out = res.cpu().tolist() + cost.cpu().tolist()
+    assert out == ref and out[0] == 0, f"sharded search {out} vs {ref}"
+    tot = [ev[0].elapsed_time(ev[4]) for ev in evs]
+    ms = pdist.max_over_ranks(statistics.mean(tot), device=dev)
+    part_ms = {k: statistics.mean([ev[i].elapsed_time(ev[i + 1]) for ev in evs])
+               for k, i in (("error_matrix_shard", 0), ("all_gather", 1), ("local_search_multi", 2), ("cost", 3))}
+    return {
+        "metric": METRIC, "value": S * S / (ms * 1e-3) / 1e9, "unit": UNIT, "n_gpus": world, "steps": K,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "u8->int32", "data": "synthetic",
+        "config": dict(workload_desc(args.config, args.family, [0]), method="trap (multi-rank)",
+                       parallelism=f"E rows sharded over {world} ranks + all-gather; Alg. 2 across ranks",
+                       l2="not flushed (E of the sharded configs exceeds L2)"),
+        "breakdown_ms_rank0": part_ms,
+        "result": {"rounds": out[1], "swaps": out[2], "cost": out[3]},
+        "clocks": clk.summary(),
+    }
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
@@ -331,6 +423,15 @@ def main():
     if world > 1:
         torch.cuda.set_device(local_rank)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    if args.sharded:
+        line = bench_sharded(args, rank, world, local_rank)
+        if rank == 0:
+            line["host"] = host_info()
+            print(json.dumps(line), flush=True)
+        if world > 1:
+            dist.barrier()
+            dist.destroy_process_group()
+        return
     line, extra = bench_ours(args, rank, world, local_rank)
     if rank == 0:
         if world == 1 and not args.no_cpu_baseline:

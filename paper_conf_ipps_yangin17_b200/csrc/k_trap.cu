@@ -697,6 +697,8 @@ struct TrapMultiParams {
   int32_t S, max_rounds, max_log, W, nchunks, world, rank0, ctas_per_rank, vec;
   LsResult* out;                  // written by the launch's first rank
   int64_t* per_round;
+  int32_t* handoff;               // the first rank's sparse-round flag (or NULL)
+  int32_t sparse_T;
 };
 
 __device__ __forceinline__ int32_t chunk_begin(int32_t r, int32_t nchunks, int32_t world) {
@@ -820,10 +822,18 @@ k_ls_trap_mr(const TrapMultiParams p) {
           }
           group_sync(1 + grp, GT);
           if (gt == 0) {
-            __threadfence_system();
-            for (int i = 0; i < nown; ++i)
-              asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p.rk[own[i]].flags + ch), "r"(q + 1u)
-                           : "memory");
+            bool remote = false;
+            for (int i = 0; i < nown; ++i) remote |= (own[i] != r);
+            if (remote) __threadfence_system();   // peer ranks: system scope
+            else __threadfence();
+            for (int i = 0; i < nown; ++i) {
+              if (own[i] != r)
+                asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p.rk[own[i]].flags + ch), "r"(q + 1u)
+                             : "memory");
+              else
+                asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.rk[own[i]].flags + ch), "r"(q + 1u)
+                             : "memory");
+            }
           }
         }
       }
@@ -858,6 +868,10 @@ k_ls_trap_mr(const TrapMultiParams p) {
     __syncthreads();
     if (rs == 0) break;
     if (p.max_rounds > 0 && rounds >= p.max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
+    if (p.handoff && rs <= p.sparse_T) {   // quiet: every rank continues alone (sparse rounds, same result)
+      if (leader && r == p.rank0) *p.handoff = 1;
+      break;
+    }
   }
   // every chunk's owned slots (class ncls - 1) into every rank's perm
   const int32_t* fin = me.rbuf[q % 3u];
@@ -910,7 +924,7 @@ size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((siz
 // Launch `nloc` ranks [rank0, rank0 + nloc) of a world on the current device.
 pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
                            int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
-                           cudaStream_t st) {
+                           cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0) {
   constexpr int PPL = 2, T = 16;
   using SM = TrapSmem<PPL, T>;
   if (S < ls_trap_min_S() || (S & 1) || world < 1 || world > kMaxRanks || nloc < 1) return PM_ERR_UNSUPPORTED;
@@ -927,6 +941,7 @@ pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_
   hp.world = world; hp.rank0 = rank0;
   hp.vec = ((int64_t)S * ldE * 4 <= (96ll << 20)) ? 1 : 0;
   hp.out = dev_out; hp.per_round = dev_per_round;
+  hp.handoff = handoff; hp.sparse_T = sparse_T;
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
   int max_cpc = (int)((size_t)optin / SM::bytes);
@@ -969,9 +984,22 @@ pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_
     PM_CUDA_TRY(cudaMemcpyAsync(pr, perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
     trap_ws_layout(ws, S, pr, E, ranks[r]);
   }
-  pm_status_t s = run_trap_multi(ranks, world, 0, world, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st);
+  // quiet rounds: every rank would continue alone with the same sparse
+  // rounds; here rank world-1 (the farthest from the launch's first) does
+  const int32_t sparse_T = ls_sparse_threshold(S, PM_LS_TRAP);
+  SparseRun sr;
+  if (sparse_T > 0) {
+    const pm_status_t s0 = sparse_prepare(E, ldE, S, ranks[world - 1].perm, max_rounds, dev_out, dev_per_round,
+                                          max_log, st, &sr);
+    if (s0 != PM_OK) return s0;
+  }
+  pm_status_t s = run_trap_multi(ranks, world, 0, world, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
+                                 sr.pending, sparse_T);
   if (s != PM_OK) return s;
-  // every rank holds the whole result; return rank world-1's (the farthest)
+  if (sparse_T > 0) {
+    const pm_status_t s1 = sparse_launch(&sr, st);
+    if (s1 != PM_OK) return s1;
+  }
   PM_CUDA_TRY(cudaMemcpyAsync(perm, ranks[world - 1].perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
   PM_CUDA_TRY(cudaFreeAsync(buf, st));
   return PM_OK;
@@ -987,6 +1015,19 @@ pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* c
   if (world < 1 || world > kMaxRanks || rank < 0 || rank >= world) return PM_ERR_INVALID;
   TrapRank ranks[kMaxRanks];
   for (int r = 0; r < world; ++r) trap_ws_layout(ws_peers[r], S, perm_peers[r], E, ranks[r]);
-  return run_trap_multi(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st);
+  // quiet rounds: this rank continues alone (sparse rounds on its own copy
+  // of r and E -- every rank reaches the same result, no exchange)
+  const int32_t sparse_T = ls_sparse_threshold(S, PM_LS_TRAP);
+  SparseRun sr;
+  if (sparse_T > 0) {
+    const pm_status_t s0 = sparse_prepare(E, ldE, S, perm_peers[rank], max_rounds, dev_out, dev_per_round, max_log,
+                                          st, &sr);
+    if (s0 != PM_OK) return s0;
+  }
+  const pm_status_t s = run_trap_multi(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
+                                       st, sr.pending, sparse_T);
+  if (s != PM_OK) return s;
+  if (sparse_T > 0) return sparse_launch(&sr, st);
+  return PM_OK;
 }
 }  // namespace pm

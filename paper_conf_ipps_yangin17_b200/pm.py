@@ -231,6 +231,11 @@ def trap_workspace_bytes(S: int) -> int:
     return int(lib().pm_trap_workspace_bytes(S))
 
 
+def trap_workspace_reset(ws, S: int, stream=None):
+    """pm_trap_workspace_reset on a CUDA byte tensor (async on the stream)."""
+    _check(lib().pm_trap_workspace_reset(ws.data_ptr(), S, _stream(stream)), "pm_trap_workspace_reset")
+
+
 def local_search_multi_async(E, perm_ptrs, ws_ptrs, rank: int, world: int, result, max_rounds: int = 0,
                              stream=None):
     """pm_local_search_multi_async: this rank's part of the multi-GPU search;
