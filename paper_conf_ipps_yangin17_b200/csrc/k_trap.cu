@@ -922,10 +922,10 @@ static void trap_ws_layout(void* ws, int32_t S, int32_t* perm, const int32_t* E,
 size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((size_t)S / 2 + 16); }
 
 // Launch `nloc` ranks [rank0, rank0 + nloc) of a world on the current device.
-pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
-                           int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
-                           cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0) {
-  constexpr int PPL = 2, T = 16;
+template <int PPL, int T>
+static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE,
+                                     int32_t S, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
+                                     int32_t max_log, cudaStream_t st, int32_t* handoff, int32_t sparse_T) {
   using SM = TrapSmem<PPL, T>;
   if (S < ls_trap_min_S() || (S & 1) || world < 1 || world > kMaxRanks || nloc < 1) return PM_ERR_UNSUPPORTED;
   int dev = 0, nsm = 0, optin = 0;
@@ -963,6 +963,20 @@ pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_
   PM_CUDA_TRY(cudaLaunchCooperativeKernel((const void*)fn, dim3(cpr * nloc), dim3(threads), args, smem, st));
   note_launch();
   return PM_OK;
+}
+
+// Chunk geometry as the single-GPU grid mode: 64 x 16 while E is
+// L2-resident or S > 16384, else 128 x 32 (PM_TRAP_V = 0 / 5 force one).
+pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
+                           int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
+                           cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0) {
+  int32_t v = trap_env("PM_TRAP_V", -1);
+  if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) ? 5 : 0;
+  if (v == 5)
+    return launch_trap_multi<4, 32>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
+                                    st, handoff, sparse_T);
+  return launch_trap_multi<2, 16>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
+                                  handoff, sparse_T);
 }
 
 

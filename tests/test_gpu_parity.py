@@ -593,6 +593,15 @@ def test_multi_rank_trap_emulated(N, M, fam, world):
     assert (rounds, swaps) == (ref[1], ref[2])
 
 
+@pytest.mark.parametrize("variant", ["0", "5"])
+def test_multi_rank_trap_geometries(variant, monkeypatch):
+    monkeypatch.setenv("PM_TRAP_V", variant)
+    E_np = oracle_E("smooth", 1024, 16)
+    ref = oracle.local_search(E_np)
+    out, rounds, swaps = pm.local_search_multi_emulated(dev(E_np), 3)
+    assert (out.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+
+
 def test_multi_rank_trap_max_rounds_then_resume():
     E_np = oracle_E("smooth", 512, 16)
     ref = oracle.local_search(E_np, max_rounds=2)
