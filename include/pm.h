@@ -64,14 +64,16 @@ typedef enum {
                           walks the classes in order, testing only those
                           classes and the pairs of already-swapped slots;
                           rounds looped on the device (CUDA-graph WHILE node) */
-  PM_LS_TRAP = 6       /* whole GPU, temporal blocking of the class sequence:
+  PM_LS_TRAP = 6       /* many SMs, temporal blocking of the class sequence:
                           pair k of class c+1 depends only on pairs k-1..k+1
-                          of class c, so a warp replays T classes on the
-                          slots of pairs [k0-T, k1+T) in shared memory (E
-                          entries staged as per-tile stride-2 runs) and
-                          writes back pairs [k0, k1); one grid barrier per
-                          T classes (persistent cooperative kernel); even
-                          S >= 256                                            */
+                          of class c, so a chunk's warps replay T classes on
+                          the slots of pairs [k0-T, k1+T) in shared memory
+                          (E entries staged as per-tile stride-2 runs) and
+                          publish pairs [k0, k1) to the neighbour chunks
+                          only: one thread-block cluster (DSMEM st.async +
+                          mbarrier, S <= 1024) or a persistent cooperative
+                          grid (per-chunk phase flags); quiet rounds then
+                          run as sparse rounds; even S >= 256 (AUTO)         */
 } pm_ls_method_t;
 
 const char* pm_status_string(pm_status_t s);

@@ -17,12 +17,20 @@
 // memory, replays the T classes on it (the valid range shrinks by one pair per
 // side and class: overlapped tiling) and publishes the slots of its owned
 // pairs.  Two modes:
-//   grid    -- persistent cooperative grid; state ping-pongs between two
-//              global buffers, one grid barrier per phase (any S).
-//   cluster -- one thread-block cluster (<= 16 CTAs) holds every chunk; each
-//              CTA keeps replicas of r and d, published slots go to the
-//              replicas of the CTAs of the neighbouring chunks by DSMEM
-//              stores, one cluster barrier per phase (small S).
+//   grid    -- persistent cooperative grid, any S; r and d in global memory.
+//              With W >= 2T a chunk writes its owned slots into buffer
+//              (q+1) mod 3 and releases a per-chunk phase flag, and waits
+//              only for its two neighbours' flags (every earlier reader of
+//              that buffer generation lies within two chunks); one grid
+//              barrier per round for the swap count.  Else one grid barrier
+//              per phase with two buffers.
+//   cluster -- one thread-block cluster (<= 16 CTAs, one chunk each) holds
+//              every chunk; each CTA keeps replicas of r and d, published
+//              slots go to the replicas of the neighbouring chunks' CTAs by
+//              st.async, completing on the receiver's mbarrier (expect_tx),
+//              one cluster barrier per round (small S).
+// The multi-rank kernel at the end of the file runs the grid mode across
+// the GPUs of one box (pm_local_search_multi_async).
 // Each pair test is line 5 with two entries carried in d (as every method
 // here): d[u] + d[v] > E[r[v]][u] + E[r[u]][v], strict (R6).
 //
