@@ -86,3 +86,23 @@ def test_edge_coloring_rejects_bad_ranges(pm):
     assert pm.lib().pm_edge_coloring(16, 0, 16, out.ctypes.data) == pm.PM_ERR_INVALID
     part = pm.edge_coloring(16, 4, 6)
     assert (part == pm.edge_coloring(16)[4:6]).all()
+
+
+def test_multi_rank_entry_points_validate_before_any_launch(pm):
+    # host-side checks of the multi-GPU boundary (no device needed)
+    import ctypes
+    L = pm.lib()
+    S = 1024
+    ws = pm.trap_workspace_bytes(S)
+    assert ws >= 5 * 4 * S and pm.trap_workspace_bytes(1) == 0
+    assert pm.trap_workspace_bytes(4 * S) > ws
+    P2 = ctypes.c_void_p * 2
+    fake = 0x1000
+    # null E / tables / result, rank outside the world, ld_E < S
+    assert L.pm_local_search_multi_async(None, S, S, P2(fake, fake), P2(fake, fake), 0, 2, 0, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_multi_async(fake, S, S, None, P2(fake, fake), 0, 2, 0, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_multi_async(fake, S, S, P2(fake, fake), P2(fake, fake), 2, 2, 0, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_multi_async(fake, S - 1, S, P2(fake, fake), P2(fake, fake), 0, 2, 0, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_multi_async(fake, S, S, P2(fake, None), P2(fake, fake), 0, 2, 0, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_trap_workspace_reset(None, S, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_multi_emulated(None, S, S, fake, 2, 0, None, None, None) == pm.PM_ERR_INVALID
