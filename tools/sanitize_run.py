@@ -13,11 +13,17 @@ for (N, M, C) in [(128, 8, 3), (90, 10, 3)]:
     assert (E.cpu().numpy() == Er).all()
     ref = oracle.local_search(Er)
     methods = os.environ.get("METHODS", "window,cta,class,pairwin").split(",")
+    perm = None
     for meth in methods:
-        if meth == "pairwin" and E.shape[0] < 40:
+        if (meth == "pairwin" and E.shape[0] < 40) or (meth == "trap" and (E.shape[0] < 256 or E.shape[0] % 2)):
             continue
         perm, rounds, swaps, per, st = pm.local_search(E, method=meth)
         assert (perm.cpu().numpy() == ref[0]).all() and rounds == ref[1], meth
+    if os.environ.get("MULTI") and E.shape[0] >= 256 and E.shape[0] % 2 == 0:
+        out, rounds, swaps = pm.local_search_multi_emulated(E, int(os.environ["MULTI"]))
+        assert (out.cpu().numpy() == ref[0]).all() and rounds == ref[1], "multi"
+    if perm is None:
+        continue
     c = pm.cost(E, perm)
     R = pm.render(dI, M, perm)
     t = pm.pack_tiles(dI, M)
