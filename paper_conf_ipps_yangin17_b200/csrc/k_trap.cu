@@ -68,6 +68,8 @@ struct TrapParams {
   int32_t W, nchunks;
   int32_t gsz;                 // warps per chunk group (= PPL)
   int32_t vec;                 // 16-byte staging allowed (PM_TRAP_VEC, default 1)
+  const int32_t* Ep;           // sigma-permuted copy of E (or NULL), leading dimension ldp
+  int64_t ldp;
   int32_t prof;                // PM_TRAP_PROF: CTA 0 thread 0 phase timers -> per_round[192..195]
   unsigned int* bar;           // grid barrier counter (zeroed before launch)
   unsigned long long* rsw;     // [3] swaps per round, rotating (grid mode)
@@ -84,6 +86,7 @@ struct TrapSmem {
   // span1 [SP, 2SP) E[g][(s0 & ~3) + q] (16-byte copies; the runs p0 + 2j,
   // s0 + 2j, j <= T, are their entries (p0 & 3) + 2j), E[g][S-1] at CL
   static constexpr int SP = (2 * T + 4 + 3) / 4 * 4;
+  static constexpr int SPP = (T + 1 + 3 + 3) / 4 * 4;   // the same runs from sigma-permuted rows
   static constexpr int CL = 2 * SP;
   static constexpr int RS = 2 * SP + 4;
   static constexpr int NC = 2 * T + 2;      // pair-0 light-cone tiles (at most)
@@ -210,7 +213,8 @@ template <int PPL, int T, typename Src>
 __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_t k1, int32_t c0, int32_t u0,
                                           const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
                                           int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
-                                          bool vec, unsigned long long* tprof) {
+                                          bool vec, unsigned long long* tprof,
+                                          const int32_t* __restrict__ Ep = nullptr, int64_t ldp = 0) {
   using SM = TrapSmem<PPL, T>;
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
@@ -228,12 +232,24 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     // p0 = partner in class c0 (the fixed tile's runs are unused)
     const int32_t p0 = fx ? u0 : wrap_m(2 * c0 + 1 - x, m);
     const int32_t s0 = fx ? u0 : x;
-    s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
-                 : make_int4(j | (2 << 16), d, j * RS + (p0 & 3), j * RS + SM::SP + (s0 & 3) + 2);
     const int32_t* row = E + (int64_t)g * ld;
     int32_t* dst = s_E + j * RS;
-    stage_span(dst, row, p0 & ~3, SM::SP, m, vec);
-    stage_span(dst + SM::SP, row, s0 & ~3, SM::SP, m, vec);
+    if (Ep) {
+      // sigma-permuted rows: Ep[g][q] = E[g][2q mod m], so the stride-2 run
+      // from column y is the contiguous run from q = sigma(y) = y (m+1)/2
+      const int32_t sp = (int32_t)(((int64_t)p0 * ((m + 1) / 2)) % m);
+      const int32_t ss = (int32_t)(((int64_t)s0 * ((m + 1) / 2)) % m);
+      s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
+                   : make_int4(j | (1 << 16), d, j * RS + (sp & 3), j * RS + SM::SP + (ss & 3) + 1);
+      const int32_t* prow = Ep + (int64_t)g * ldp;
+      for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + q, prow + (sp & ~3) + q);
+      for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + SM::SP + q, prow + (ss & ~3) + q);
+    } else {
+      s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
+                   : make_int4(j | (2 << 16), d, j * RS + (p0 & 3), j * RS + SM::SP + (s0 & 3) + 2);
+      stage_span(dst, row, p0 & ~3, SM::SP, m, vec);
+      stage_span(dst + SM::SP, row, s0 & ~3, SM::SP, m, vec);
+    }
     cp_async4(dst + SM::CL, row + (S - 1));
     if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, vec);
   }
@@ -373,7 +389,7 @@ k_ls_trap(const TrapParams p) {
             const int2* rr = rep + cur * S;
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { const int2 v = rr[x]; g = v.x; d = v.y; },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp);
           } else {
             const int bi = p.nbsync ? (int)(qph % 3u) : cur;
             const int32_t* __restrict__ rc = bi == 0 ? p.rbuf[0] : (bi == 1 ? p.rbuf[1] : p.rbuf[2]);
@@ -397,7 +413,7 @@ k_ls_trap(const TrapParams p) {
             }
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
           // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
@@ -649,6 +665,16 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.bar = bar; hp.rsw = rsw;
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.prof = trap_env("PM_TRAP_PROF", 0);
+  // sigma-permuted rows while E is L2-resident (the runs become contiguous:
+  // 5 instead of 9 16-byte pieces per run at T = 16)
+  int32_t* Ep = nullptr;
+  if ((int64_t)S * ldE * 4 <= (96ll << 20) && trap_env("PM_TRAP_EP", 1)) {
+    const int32_t m = S - 1, ext = 48;   // >= SPP + 4 for every T used
+    const int64_t ldp = ((int64_t)m + ext + 31) / 32 * 32;
+    PM_CUDA_TRY(pm::scratch_alloc(&Ep, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
+    PM_CUDA_TRY(launch_permute_cols(E, ldE, Ep, ldp, S, m, ext, st));
+    hp.Ep = Ep; hp.ldp = ldp;
+  }
   // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
   // used runs win (config 4: 5.0 vs 10.8 us)
@@ -671,6 +697,7 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
       break;
   }
   if (s != PM_OK) return s;
+  if (Ep) PM_CUDA_TRY(cudaFreeAsync(Ep, st));
   PM_CUDA_TRY(cudaFreeAsync(scratch, st));
   return PM_OK;
 }
