@@ -633,3 +633,14 @@ def test_multi_rank_trap_symmetric_memory_world1():
     finally:
         if own:
             tdist.destroy_process_group()
+
+
+@pytest.mark.parametrize("ep,mode", [("0", "1"), ("0", "0"), ("1", "0"), ("1", "1")])
+def test_trap_sigma_permuted_and_plain_row_staging(ep, mode, monkeypatch):
+    # runs staged from the sigma-permuted copy of E (default while E is
+    # L2-resident) or from E's rows directly: identical results
+    monkeypatch.setenv("PM_TRAP_EP", ep)
+    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
+    monkeypatch.setenv("PM_LS_SPARSE", "0")
+    _check_trap(oracle_E("smooth", 512, 16))
+    _check_trap(oracle_E("ties", 128, 8))
