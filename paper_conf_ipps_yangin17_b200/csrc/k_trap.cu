@@ -725,10 +725,11 @@ struct TrapRank {                 // one rank's workspace (see trap_ws_layout)
   unsigned long long* rtot;       // [3] round swap totals (all ranks add)
   int32_t* perm;
   const int32_t* E;
+  const int32_t* Ep;              // this rank's sigma-permuted copy of E (or NULL)
 };
 struct TrapMultiParams {
   TrapRank rk[kMaxRanks];
-  int64_t ldE;
+  int64_t ldE, ldp;
   int32_t S, max_rounds, max_log, W, nchunks, world, rank0, ctas_per_rank, vec;
   LsResult* out;                  // written by the launch's first rank
   int64_t* per_round;
@@ -830,7 +831,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
           const int32_t* __restrict__ dc = me.dbuf[bi];
           mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                      [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
-                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr);
+                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp);
           // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
           int32_t own[3];
           int nown = 0;
@@ -953,6 +954,7 @@ static void trap_ws_layout(void* ws, int32_t S, int32_t* perm, const int32_t* E,
   rk.dbuf[0] = base + 2 * n; rk.dbuf[1] = base + 3 * n; rk.dbuf[2] = base + 4 * n;
   rk.perm = perm;
   rk.E = E;
+  rk.Ep = nullptr;
 }
 size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((size_t)S / 2 + 16); }
 
@@ -960,7 +962,8 @@ size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((siz
 template <int PPL, int T>
 static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE,
                                      int32_t S, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
-                                     int32_t max_log, cudaStream_t st, int32_t* handoff, int32_t sparse_T) {
+                                     int32_t max_log, cudaStream_t st, int32_t* handoff, int32_t sparse_T,
+                                     int64_t ldp) {
   using SM = TrapSmem<PPL, T>;
   if (S < ls_trap_min_S() || (S & 1) || world < 1 || world > kMaxRanks || nloc < 1) return PM_ERR_UNSUPPORTED;
   int dev = 0, nsm = 0, optin = 0;
@@ -977,6 +980,7 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   hp.vec = ((int64_t)S * ldE * 4 <= (96ll << 20)) ? 1 : 0;
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.handoff = handoff; hp.sparse_T = sparse_T;
+  hp.ldp = ldp;
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
   int max_cpc = (int)((size_t)optin / SM::bytes);
@@ -1004,16 +1008,29 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
 // L2-resident or S > 16384, else 128 x 32 (PM_TRAP_V = 0 / 5 force one).
 pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
                            int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
-                           cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0) {
+                           cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0, int64_t ldp = 0) {
   int32_t v = trap_env("PM_TRAP_V", -1);
   if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) ? 5 : 0;
   if (v == 5)
     return launch_trap_multi<4, 32>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
-                                    st, handoff, sparse_T);
+                                    st, handoff, sparse_T, ldp);
   return launch_trap_multi<2, 16>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
-                                  handoff, sparse_T);
+                                  handoff, sparse_T, ldp);
 }
 
+
+// sigma-permuted copy of E while it is L2-resident (as run_trap); NULL else.
+static pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
+                                 int64_t* ldp) {
+  *Ep = nullptr;
+  *ldp = 0;
+  if ((int64_t)S * ldE * 4 > (96ll << 20) || !trap_env("PM_TRAP_EP", 1)) return PM_OK;
+  const int32_t m = S - 1, ext = 48;
+  *ldp = ((int64_t)m + ext + 31) / 32 * 32;
+  PM_CUDA_TRY(pm::scratch_alloc(Ep, sizeof(int32_t) * (size_t)S * (size_t)*ldp, st));
+  PM_CUDA_TRY(launch_permute_cols(E, ldE, *Ep, *ldp, S, m, ext, st));
+  return PM_OK;
+}
 
 // All ranks of a world on the current device, one launch (test hook).
 pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
@@ -1042,9 +1059,17 @@ pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_
                                           max_log, st, &sr);
     if (s0 != PM_OK) return s0;
   }
+  int32_t* Ep = nullptr;
+  int64_t ldp = 0;
+  {
+    const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+    if (se != PM_OK) return se;
+  }
+  for (int r = 0; r < world; ++r) ranks[r].Ep = Ep;
   pm_status_t s = run_trap_multi(ranks, world, 0, world, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
-                                 sr.pending, sparse_T);
+                                 sr.pending, sparse_T, ldp);
   if (s != PM_OK) return s;
+  if (Ep) PM_CUDA_TRY(cudaFreeAsync(Ep, st));
   if (sparse_T > 0) {
     const pm_status_t s1 = sparse_launch(&sr, st);
     if (s1 != PM_OK) return s1;
@@ -1073,9 +1098,17 @@ pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* c
                                           st, &sr);
     if (s0 != PM_OK) return s0;
   }
+  int32_t* Ep = nullptr;
+  int64_t ldp = 0;
+  {
+    const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+    if (se != PM_OK) return se;
+  }
+  ranks[rank].Ep = Ep;   // only this rank's entry is read by this launch
   const pm_status_t s = run_trap_multi(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
-                                       st, sr.pending, sparse_T);
+                                       st, sr.pending, sparse_T, ldp);
   if (s != PM_OK) return s;
+  if (Ep) PM_CUDA_TRY(cudaFreeAsync(Ep, st));
   if (sparse_T > 0) return sparse_launch(&sr, st);
   return PM_OK;
 }
