@@ -665,10 +665,14 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.bar = bar; hp.rsw = rsw;
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.prof = trap_env("PM_TRAP_PROF", 0);
-  // sigma-permuted rows while E is L2-resident (the runs become contiguous:
-  // 5 instead of 9 16-byte pieces per run at T = 16)
+  // sigma-permuted rows (the runs become contiguous: 5 instead of 9 16-byte
+  // pieces per run at T = 16 from L2, dense sectors instead of stride-2 ones
+  // from HBM)
   int32_t* Ep = nullptr;
-  if ((int64_t)S * ldE * 4 <= (96ll << 20) && trap_env("PM_TRAP_EP", 1)) {
+  // (measured: config 2 1.25 -> 1.18 ms, config 4 67.4 -> 62.3 ms; config 5
+  // 1.09 -> 1.25 s -- building the 16 GiB copy costs more than it saves)
+  const int32_t ep_mode = trap_env("PM_TRAP_EP", 1);   // 0 off, 1 up to E = 2 GiB, 2 always
+  if (ep_mode == 2 || ((int64_t)S * ldE * 4 <= (2ll << 30) && ep_mode == 1)) {
     const int32_t m = S - 1, ext = 48;   // >= SPP + 4 for every T used
     const int64_t ldp = ((int64_t)m + ext + 31) / 32 * 32;
     PM_CUDA_TRY(pm::scratch_alloc(&Ep, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
@@ -1019,12 +1023,13 @@ pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_
 }
 
 
-// sigma-permuted copy of E while it is L2-resident (as run_trap); NULL else.
+// sigma-permuted copy of E up to E = 2 GiB (as run_trap); NULL else.
 static pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
                                  int64_t* ldp) {
   *Ep = nullptr;
   *ldp = 0;
-  if ((int64_t)S * ldE * 4 > (96ll << 20) || !trap_env("PM_TRAP_EP", 1)) return PM_OK;
+  const int32_t ep_mode = trap_env("PM_TRAP_EP", 1);
+  if (ep_mode == 0 || (ep_mode == 1 && (int64_t)S * ldE * 4 > (2ll << 30))) return PM_OK;
   const int32_t m = S - 1, ext = 48;
   *ldp = ((int64_t)m + ext + 31) / 32 * 32;
   PM_CUDA_TRY(pm::scratch_alloc(Ep, sizeof(int32_t) * (size_t)S * (size_t)*ldp, st));
