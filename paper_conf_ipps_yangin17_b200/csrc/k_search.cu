@@ -364,17 +364,20 @@ __global__ void __launch_bounds__(256) k_cost(const int32_t* __restrict__ E, int
   if (threadIdx.x == 0) {
     long long t = 0;
     for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
-    atomicAdd(cost, (unsigned long long)t);
+    if (gridDim.x == 1) *cost = (unsigned long long)t;   // one block: no zeroing, no atomic
+    else atomicAdd(cost, (unsigned long long)t);
   }
 }
 
 cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm, int64_t* d_cost,
                         cudaStream_t st) {
-  cudaError_t e = cudaMemsetAsync(d_cost, 0, sizeof(int64_t), st);
-  if (e != cudaSuccess) return e;
-  int blocks = (S + 255) / 256;
+  int blocks = (S + 2047) / 2048;   // <= 8 gathers per thread
   if (blocks < 1) blocks = 1;
   if (blocks > 148) blocks = 148;
+  if (blocks > 1) {
+    cudaError_t e = cudaMemsetAsync(d_cost, 0, sizeof(int64_t), st);
+    if (e != cudaSuccess) return e;
+  }
   k_cost<<<blocks, 256, 0, st>>>(E, ldE, S, perm, reinterpret_cast<unsigned long long*>(d_cost));
   note_launch();
   return cudaGetLastError();
