@@ -374,22 +374,29 @@ pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
   const int32_t g = N / M;
   const int64_t S = (int64_t)g * g;
   const size_t img = (size_t)N * N * C;
-  const size_t bytes = 2 * img + sizeof(int32_t) * (size_t)S * (size_t)S + sizeof(int32_t) * (size_t)S + 64;
+  const size_t bytes = 64 + 2 * img + sizeof(int32_t) * (size_t)S * (size_t)S + sizeof(int32_t) * (size_t)S + 64;
   DevBuf buf;
   buf.st = st;
   PM_CUDA_TRY(pm::scratch_alloc(&buf.p, bytes, st));
   char* base = reinterpret_cast<char*>(buf.p);
-  int32_t* dE = reinterpret_cast<int32_t*>(base);
+  int64_t* dres = reinterpret_cast<int64_t*>(base);          // {status, rounds, swaps, cost}
+  int32_t* dE = reinterpret_cast<int32_t*>(base + 64);
   int32_t* dperm = dE + S * S;
   uint8_t* dI = reinterpret_cast<uint8_t*>(dperm + S);
   uint8_t* dT = dI + img;
   PM_CUDA_TRY(cudaMemcpyAsync(dI, h_input, img, cudaMemcpyHostToDevice, st));
   PM_CUDA_TRY(cudaMemcpyAsync(dT, h_target, img, cudaMemcpyHostToDevice, st));
-  pm_status_t s = pm_photomosaic(dI, dT, N, M, C, dE, S, dperm, method, h_rounds, h_swaps, h_cost, stream);
+  pm_status_t s = pm_photomosaic_async(dI, dT, N, M, C, dE, S, dperm, method, dres, stream);
   if (s != PM_OK) return s;
+  // the result and r back in stream order, one host synchronisation
+  int64_t h[4];
   PM_CUDA_TRY(cudaMemcpyAsync(h_perm, dperm, sizeof(int32_t) * (size_t)S, cudaMemcpyDeviceToHost, st));
+  PM_CUDA_TRY(cudaMemcpyAsync(h, dres, sizeof(h), cudaMemcpyDeviceToHost, st));
   PM_CUDA_TRY(cudaStreamSynchronize(st));
-  return PM_OK;
+  if (h_rounds) *h_rounds = (int32_t)h[1];
+  if (h_swaps) *h_swaps = h[2];
+  if (h_cost) *h_cost = h[3];
+  return (pm_status_t)h[0];
 }
 
 pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, const int32_t* d_perm,
