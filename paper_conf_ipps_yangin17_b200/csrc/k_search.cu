@@ -353,9 +353,19 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
 __global__ void __launch_bounds__(256) k_cost(const int32_t* __restrict__ E, int64_t ld, int32_t S,
                                               const int32_t* __restrict__ perm,
                                               unsigned long long* __restrict__ cost) {
+  // up to 8 gathers per thread, all r loads then all E loads in flight (two
+  // memory round trips instead of one per gather)
+  constexpr int U = 8;
   long long s = 0;
-  for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < S; u += gridDim.x * blockDim.x)
-    s += __ldg(E + (int64_t)__ldg(perm + u) * ld + u);
+  const int32_t stride = gridDim.x * blockDim.x;
+  for (int32_t u0 = blockIdx.x * blockDim.x + threadIdx.x; u0 < S; u0 += U * stride) {
+    int32_t rq[U];
+#pragma unroll
+    for (int q = 0; q < U; ++q) rq[q] = (u0 + q * stride < S) ? __ldg(perm + u0 + q * stride) : -1;
+#pragma unroll
+    for (int q = 0; q < U; ++q)
+      if (rq[q] >= 0) s += __ldg(E + (int64_t)rq[q] * ld + (u0 + q * stride));
+  }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   __shared__ long long red[8];
