@@ -11,9 +11,10 @@
  *   - stream : a cudaStream_t (NULL = legacy default stream).  Device work is
  *     enqueued on it; functions that return host scalars synchronise it.
  *   - Ownership: the caller allocates and frees every buffer it passes.  The
- *     library keeps no state between calls except cached, immutable launch
- *     plans; scratch memory comes from cudaMallocAsync on `stream` and is
- *     freed before return.
+ *     library keeps no state between calls except cached launch plans and
+ *     its scratch pool; scratch comes from a stream-ordered pool on
+ *     `stream` and is freed (to the pool) before return -- see
+ *     pm_scratch_trim for what the pool keeps.
  *   - Errors: every argument is validated before any launch
  *     (PM_ERR_INVALID, nothing enqueued).  CUDA failures map to PM_ERR_CUDA.
  *     No C++ exception crosses this boundary.  Outputs are undefined on error.
@@ -40,24 +41,23 @@ typedef enum {
   PM_ERR_CUDA = 2,           /* a CUDA runtime call or launch failed          */
   PM_ERR_NOT_CONVERGED = 3,  /* max_rounds reached before a zero-swap round   */
   PM_ERR_UNSUPPORTED = 4,    /* valid, but outside what this build supports   */
-  PM_ERR_NOT_PERMUTATION = 5 /* d_perm is not a bijection of [0, S)    */
+  PM_ERR_NOT_PERMUTATION = 5, /* d_perm is not a bijection of [0, S)   */
+  PM_ERR_TIMEOUT = 6         /* multi-GPU: a peer rank did not arrive within
+                                the wait limit (pm_local_search_multi_async) */
 } pm_status_t;
 
-/* Local-search implementation selector for pm_local_search_ex. */
+/* Local-search implementation selector for pm_local_search_ex.  Every method
+ * returns the same r, rounds and per-round swaps (Alg. 2 is deterministic
+ * under readings R5-R10); they differ only in speed and in the S they take.
+ * Values 2 and 4 (the single-CTA and pair-window methods of round 1,
+ * dominated on every S) are retired: PM_ERR_INVALID. */
 typedef enum {
   PM_LS_AUTO = 0,      /* pick the fastest method supported for S            */
   PM_LS_CLASS = 1,     /* one kernel per colour class P_i, the paper's own
                           launch structure, replayed as a CUDA graph  */
-  PM_LS_CTA = 2,       /* one CTA runs every round on the device: r and the
-                          maintained diagonal d in shared memory, E gathered
-                          from L2/HBM (S <= pm_ls_cta_max_S())                */
   PM_LS_WINDOW = 3,    /* one CTA, plus a shared-memory window of each slot's
-                          upcoming E entries streamed ahead of the classes    */
-  PM_LS_PAIRWIN = 4,   /* per round: a grid-wide kernel tabulates every pair's
-                          two terms of line 5 at the round's start, one CTA
-                          streams the class rows and patches swapped slots;
-                          rounds looped on the device (CUDA-graph WHILE node);
-                          40 <= S <= 2048 on this build                       */
+                          upcoming E entries streamed ahead of the classes
+                          (S <= 2048)                                         */
   PM_LS_WALK = 5,      /* every round as a sparse round: a whole-GPU test of
                           every pair on the round's start state marks the
                           classes that can fire, then a thread-block cluster
@@ -191,7 +191,11 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
  *   pm_local_search_multi_emulated : test hook -- all `world` ranks in one
  *            launch on the current device (own workspaces and perms), the
  *            exchange protocol unchanged; d_perm in/out as pm_local_search.
- * world <= 8; S even, >= 256, and S/64 >= world. */
+ * world <= 8; S even, >= 256, and at least `world` pair chunks (S/64 chunks
+ * while E is L2-resident or S > 16384, else S/128): else PM_ERR_UNSUPPORTED,
+ * before anything is enqueued.  Every cross-GPU wait is bounded (20 s): a
+ * rank whose peer never arrives stops and reports PM_ERR_TIMEOUT in
+ * d_result (d_perm is then unspecified on that rank). */
 size_t pm_trap_workspace_bytes(int32_t S);
 pm_status_t pm_trap_workspace_reset(void* d_ws, int32_t S, pm_stream_t stream);
 pm_status_t pm_local_search_multi_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* const* d_perm_peers,
@@ -203,10 +207,6 @@ pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int
 
 /* The method PM_LS_AUTO selects for S on the current device (host-only). */
 int32_t pm_ls_auto_method(int32_t S);
-
-/* Largest S the single-CTA methods accept on this device (shared-memory
- * bound); 0 if no device. */
-int32_t pm_ls_cta_max_S(void);
 
 /* r := identity (Alg. 1/2 start from the input image as given, P:116-120,
  * reading R7).  d_perm : int32 [S].  Async on stream. */
@@ -283,10 +283,41 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
 
 /* Number of this library's kernel launches by the calling process so far
  * (for launch accounting in benchmarks): host-side launches plus the kernels
- * that device-side graph loops (CLASS / PAIRWIN rounds, sparse rounds)
+ * that device-side graph loops (CLASS rounds, sparse rounds)
  * launched, which count themselves on the device -- so this call reads a
  * device counter back and synchronises with the devices it has used. */
 int64_t pm_launch_count(void);
+
+/* Tuning overrides, for tests and development tools only.  Every method
+ * reads its geometry and hand-over choices from measured defaults; these
+ * calls override one of them process-wide (never read from the
+ * environment).  Results stay bit-exact under every override -- only speed
+ * and the set of supported S change (an override that a launch cannot honour
+ * returns PM_ERR_UNSUPPORTED from the search).
+ *   name  : one of "trap_variant" (chunk geometry 0..5), "trap_W" (owned
+ *           pairs per chunk), "trap_cluster" (0 grid, 1 cluster), "trap_nbsync",
+ *           "trap_cpc", "trap_ep" (sigma-permuted staging: 0 off, 1 auto,
+ *           2 always), "trap_vec", "trap_spec", "trap_prefetch", "trap_prof",
+ *           "trap_wait_ms" (bound of the multi-GPU waits, default 20000),
+ *           "ls_sparse" (0: no sparse rounds), "ls_sparse_T" (hand-over swap
+ *           count), "ls_cwalk" (0 one-CTA walk, 1 cluster walk),
+ *           "ls_sparse_gmem", "auction_gs", "auction_keep",
+ *           "auction_smem_price", "auction_theta", "auction_eps_shift",
+ *           "auction_max_rounds", "auction_ctas_per_sm".
+ * PM_ERR_INVALID for an unknown name.  pm_tuning_reset restores every
+ * default.  Not synchronised with searches running on other threads. */
+pm_status_t pm_tuning_set(const char* name, int32_t value);
+void pm_tuning_reset(void);
+
+/* Scratch.  Every call takes its scratch from a library-owned stream-ordered
+ * pool on the current device and frees it before returning (in stream
+ * order).  The pool keeps up to 4 GiB mapped between calls so repeated calls
+ * do not re-map memory; memory beyond that returns to the driver at the next
+ * synchronisation.  pm_scratch_trim releases everything the pool holds that
+ * no pending work uses (call after synchronising the streams used);
+ * pm_scratch_reserved_bytes reports what the pool holds now. */
+pm_status_t pm_scratch_trim(void);
+size_t pm_scratch_reserved_bytes(void);
 
 #ifdef __cplusplus
 }

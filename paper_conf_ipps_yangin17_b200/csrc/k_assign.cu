@@ -325,11 +325,6 @@ __global__ void __launch_bounds__(kThreads) k_auction(AuctionArgs a) {
   if (gtid == 0) ctr[kCLen0] = n_u;             // unassigned at exit (0 = converged)
 }
 
-static int env_int(const char* name, int dflt) {
-  const char* v = getenv(name);
-  return v ? atoi(v) : dflt;
-}
-
 // Exact optimum of sum_v E[r[v]][v] over bijections r (Eq. 3, P:70 / P:98).
 pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* perm, int64_t* price_out,
                            int64_t* cost_out_dev, int32_t* h_stats, cudaStream_t st) {
@@ -345,12 +340,12 @@ pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* per
   PM_CUDA_TRY(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   const size_t static_smem = 8 * 1024;        // s_best, s_q and headroom
   const size_t dyn = (size_t)S * (sizeof(int64_t) + sizeof(int32_t));
-  const bool smem_price = env_int("PM_AUCTION_SMEM_PRICE", 1) && dyn + static_smem <= (size_t)smem_optin;
+  const bool smem_price = knob("auction_smem_price", 1) && dyn + static_smem <= (size_t)smem_optin;
   const size_t dyn_bytes = smem_price ? dyn : 0;
   PM_CUDA_TRY(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn_bytes));
   PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, kThreads, dyn_bytes));
   if (per_sm < 1) return PM_ERR_UNSUPPORTED;
-  const int cap = env_int("PM_AUCTION_CTAS_PER_SM", 1);
+  const int cap = knob("auction_ctas_per_sm", 1);
   int blocks = sms * (per_sm < cap ? per_sm : cap);
 
   char* buf = nullptr;
@@ -365,12 +360,12 @@ pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* per
   a.myobj = a.owner + S;
   a.list = a.myobj + S;
   a.counters = a.list + 2 * (size_t)S;
-  a.theta = env_int("PM_AUCTION_THETA", 8);
-  a.eps_shift = env_int("PM_AUCTION_EPS_SHIFT", 3);
-  a.max_rounds = env_int("PM_AUCTION_MAX_ROUNDS", 1 << 22);
-  a.gs_threshold = env_int("PM_AUCTION_GS", 8);
+  a.theta = knob("auction_theta", 8);
+  a.eps_shift = knob("auction_eps_shift", 3);
+  a.max_rounds = knob("auction_max_rounds", 1 << 22);
+  a.gs_threshold = knob("auction_gs", 8);
   a.smem_price = smem_price;
-  a.keep_pairs = env_int("PM_AUCTION_KEEP", 0);
+  a.keep_pairs = knob("auction_keep", 0);
   if (a.theta < 2) a.theta = 2;
   if (a.gs_threshold < 0) a.gs_threshold = 0;
   if (a.gs_threshold > kGsMax) a.gs_threshold = kGsMax;
@@ -386,10 +381,6 @@ pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* per
   PM_CUDA_TRY(cudaStreamSynchronize(st));
   PM_CUDA_TRY(cudaFreeAsync(buf, st));
   if (h_stats) { h_stats[0] = hc[kCRounds]; h_stats[1] = hc[kCPhases]; }
-  if (getenv("PM_AUCTION_DEBUG"))
-    fprintf(stderr, "auction S=%d blocks=%d vec=%d steps=%d phases=%d gs_bids=%d jacobi n_u hist <=1:%d <=4:%d <=16:%d <=64:%d >64:%d\n",
-            S, blocks, (int)vec, hc[kCRounds], hc[kCPhases], hc[kCGsBids], hc[kCHist], hc[kCHist + 1], hc[kCHist + 2],
-            hc[kCHist + 3], hc[kCHist + 4]);
   if (hc[kCBad]) return PM_ERR_INVALID;
   if (hc[kCLen0] != 0) return PM_ERR_NOT_CONVERGED;
   if (cost_out_dev) PM_CUDA_TRY(launch_cost(E, ld, S, perm, cost_out_dev, st));

@@ -13,8 +13,6 @@
 //             n-1 class launches of a round captured once into a CUDA graph
 //             whose while-node repeats rounds on the device until a round
 //             has no swap (no host round trip per round).
-//   CTA    -- one CTA runs every round: r and d in shared memory, a
-//             __syncthreads() between classes instead of a kernel boundary.
 #include <cuda_runtime.h>
 
 #include <map>
@@ -115,8 +113,12 @@ struct ClassGraph {
   cudaGraphExec_t exec = nullptr;
 };
 
-static std::mutex g_graph_mu;
-static std::map<std::tuple<int, int32_t, cudaStream_t>, ClassGraph> g_graphs;
+// One cache per host thread (a cached graph reads one device params struct,
+// so two threads sharing a stream handle -- the legacy default stream,
+// cudaStreamPerThread -- must not share an entry); bounded: beyond
+// kGraphCacheMax entries the thread's cache is dropped after a device sync.
+constexpr size_t kGraphCacheMax = 64;
+static thread_local std::map<std::tuple<int, int32_t, cudaStream_t>, ClassGraph> g_graphs;
 
 static cudaError_t build_class_graph(int32_t S, cudaStream_t st, ClassGraph& out) {
   const Classes cl(S);
@@ -160,9 +162,16 @@ static pm_status_t run_class(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   PM_CUDA_TRY(cudaGetDevice(&dev));
   ClassGraph cg;
   {
-    std::lock_guard<std::mutex> lk(g_graph_mu);
     auto key = std::make_tuple(dev, S, st);
     auto it = g_graphs.find(key);
+    if (it == g_graphs.end() && g_graphs.size() >= kGraphCacheMax) {
+      PM_CUDA_TRY(cudaDeviceSynchronize());
+      for (auto& kv : g_graphs) {
+        cudaGraphExecDestroy(kv.second.exec);
+        cudaFree(kv.second.dparams);
+      }
+      g_graphs.clear();
+    }
     if (it == g_graphs.end()) {
       ClassGraph ng;
       PM_CUDA_TRY(build_class_graph(S, st, ng));
@@ -191,119 +200,22 @@ static pm_status_t run_class(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   return PM_OK;
 }
 
-// --------------------------------------------------------------- CTA -----
-// One CTA, kThreads threads, runs Algorithm 2 to convergence.  Dynamic smem:
-// r [S] and d [S] (int32) + a small reduction area.
-constexpr int kCtaThreads = 1024;
-
-__device__ __forceinline__ int block_sum(int v, int* s_red) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
-  __syncthreads();
-  if (l == 0) s_red[w] = v;
-  __syncthreads();
-  int t = 0;
-  if (threadIdx.x < 32) {
-    t = (threadIdx.x < (blockDim.x >> 5)) ? s_red[threadIdx.x] : 0;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
-    if (threadIdx.x == 0) s_red[32] = t;
-  }
-  __syncthreads();
-  return s_red[32];
-}
-
-__global__ void __launch_bounds__(kCtaThreads, 1)
-k_ls_cta(const int32_t* __restrict__ E, int64_t ld, int32_t S, int32_t* __restrict__ perm,
-         int32_t max_rounds, LsResult* out, int64_t* per_round, int32_t max_log) {
-  extern __shared__ int32_t sm[];
-  int32_t* s_r = sm;
-  int32_t* s_d = sm + S;
-  int* s_red = sm + 2 * S;        // 33 ints
-  const Classes cl(S);
-  const int T = blockDim.x;
-
-  // Permutation check (r is a bijection), then d[u] = E[r[u]][u].
-  for (int32_t x = threadIdx.x; x < S; x += T) s_d[x] = 0;
-  __syncthreads();
-  int bad = 0;
-  for (int32_t u = threadIdx.x; u < S; u += T) {
-    const int32_t t = perm[u];
-    s_r[u] = t;
-    if (t < 0 || t >= S) bad = 1;
-    else atomicAdd(&s_d[t], 1);
-  }
-  __syncthreads();
-  for (int32_t x = threadIdx.x; x < S; x += T)
-    if (s_d[x] != 1) bad = 1;
-  if (__syncthreads_or(bad)) {
-    if (threadIdx.x == 0) { out->status = PM_ERR_NOT_PERMUTATION; out->rounds = 0; out->swaps = 0; }
-    return;
-  }
-  for (int32_t u = threadIdx.x; u < S; u += T) s_d[u] = __ldg(E + (int64_t)s_r[u] * ld + u);
-  __syncthreads();
-
-  int32_t rounds = 0;
-  int64_t total = 0;
-  int status = PM_OK;
-  for (;;) {
-    int mysw = 0;
-    for (int32_t c = 0; c < cl.ncls; ++c) {
-      for (int32_t k = threadIdx.x; k < cl.npairs; k += T) {
-        int32_t u, v;
-        cl.pair(c, k, u, v);
-        const int32_t a = s_r[u], b = s_r[v];
-        const int32_t e_bu = __ldg(E + (int64_t)b * ld + u);
-        const int32_t e_av = __ldg(E + (int64_t)a * ld + v);
-        const int32_t du = s_d[u], dv = s_d[v];
-        if ((int64_t)du + dv > (int64_t)e_bu + e_av) {
-          s_r[u] = b; s_r[v] = a;
-          s_d[u] = e_bu; s_d[v] = e_av;
-          ++mysw;
-        }
-      }
-      __syncthreads();
-    }
-    const int sw = block_sum(mysw, s_red);
-    if (threadIdx.x == 0 && rounds < max_log) per_round[rounds] = sw;
-    rounds += 1;
-    total += sw;
-    if (sw == 0) break;
-    if (max_rounds > 0 && rounds >= max_rounds) { status = PM_ERR_NOT_CONVERGED; break; }
-  }
-  for (int32_t u = threadIdx.x; u < S; u += T) perm[u] = s_r[u];
-  if (threadIdx.x == 0) { out->status = status; out->rounds = rounds; out->swaps = total; }
-}
-
-static int32_t cta_smem_bytes(int32_t S) { return (int32_t)(sizeof(int32_t) * (2 * (size_t)S + 40)); }
-
-int32_t ls_cta_max_S() {
-  int dev = 0, optin = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
-  if (cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) return 0;
-  return (int32_t)((optin / 4 - 40) / 2);
-}
-
-static pm_status_t run_cta(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
-                           LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
-  const int32_t smem = cta_smem_bytes(S);
-  PM_CUDA_TRY(cudaFuncSetAttribute(k_ls_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  int threads = kCtaThreads;
-  while (threads > 64 && threads / 2 >= (S / 2)) threads /= 2;   // small S: fewer idle warps
-  k_ls_cta<<<1, threads, smem, st>>>(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log);
-  note_launch();
-  PM_CUDA_TRY(cudaGetLastError());
+pm_status_t ls_method_supported(int32_t S, int32_t method) {
+  if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
+  if (method == PM_LS_TRAP && (S < ls_trap_min_S() || (S & 1))) return PM_ERR_UNSUPPORTED;
+  if (method == PM_LS_WINDOW && S > ls_window_max_S()) return PM_ERR_UNSUPPORTED;
   return PM_OK;
 }
 
 pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                              int32_t method, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                              cudaStream_t st, int32_t* used_method) {
-  const int32_t cta_max = ls_cta_max_S();
   if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
   if (used_method) *used_method = method;
-  if (method == PM_LS_TRAP && (S < ls_trap_min_S() || (S & 1))) return PM_ERR_UNSUPPORTED;
+  {
+    const pm_status_t v = ls_method_supported(S, method);
+    if (v != PM_OK) return v;
+  }
   const int32_t sparse_T = (method == PM_LS_CLASS || method == PM_LS_WINDOW || method == PM_LS_TRAP)
                                ? ls_sparse_threshold(S, method) : 0;
   SparseRun sr;
@@ -316,9 +228,6 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
     case PM_LS_CLASS:
       s = run_class(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
       break;
-    case PM_LS_CTA:
-      if (S > cta_max) return PM_ERR_UNSUPPORTED;
-      return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     case PM_LS_TRAP:
       s = run_trap(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
       break;
@@ -326,16 +235,15 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
       s = run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
       break;
     case PM_LS_WALK: {
-      // every round a sparse round: start-state scan + cluster walk (S >= 2)
-      if (S < 2) return run_cta(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
+      // every round a sparse round: start-state scan + cluster walk (S >= 2;
+      // S = 1 has no colour class: one empty round, as the class graph runs it)
+      if (S < 2) return run_class(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, nullptr, 0);
       PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
       SparseRun wr;
       const pm_status_t s0 = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &wr, 1);
       if (s0 != PM_OK) return s0;
       return sparse_launch(&wr, st);
     }
-    case PM_LS_PAIRWIN:
-      return run_pairwin(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st);
     default:
       return PM_ERR_UNSUPPORTED;
   }

@@ -448,8 +448,9 @@ struct SpGraph {
   cudaGraphExec_t exec = nullptr;
 };
 
-static std::mutex g_sp_mu;
-static std::map<std::tuple<int, int32_t, cudaStream_t, bool, bool>, SpGraph> g_sp_graphs;
+// Per host thread and bounded, as the CLASS graph cache (k_search.cu).
+constexpr size_t kSpCacheMax = 64;
+static thread_local std::map<std::tuple<int, int32_t, cudaStream_t, bool, bool>, SpGraph> g_sp_graphs;
 
 static int scan_blocks(int32_t S) {
   const int64_t total = (int64_t)Classes(S).ncls * Classes(S).npairs;
@@ -513,14 +514,9 @@ static cudaError_t build_sparse_graph(int32_t S, bool use_smem, bool cluster, Sp
   return e;
 }
 
-static int32_t env_or(const char* name, int32_t dflt) {
-  const char* v = getenv(name);
-  return v ? (int32_t)atoi(v) : dflt;
-}
-
 int32_t ls_sparse_threshold(int32_t S, int32_t dense_method) {
-  if (S < 2 || !env_or("PM_LS_SPARSE", 1)) return 0;
-  const int32_t t = env_or("PM_LS_SPARSE_T", -1);
+  if (S < 2 || !knob("ls_sparse", 1)) return 0;
+  const int32_t t = knob("ls_sparse_T", -1);
   if (t >= 0) return t;
   // measured on B200: S <= 2048 (WINDOW + one-CTA walk): a
   // sparse round costs ~2 windows of ~1.3 us per swap plus ~15 us, a WINDOW
@@ -548,15 +544,22 @@ pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* pe
   // the walk: one CTA for S <= 2048, a thread-block cluster (k_cwalk.cu)
   // beyond (measured: its cluster barrier per window only pays once the dirty
   // sets outgrow one CTA); PM_LS_CWALK=0/1 forces either
-  const int32_t cw_env = env_or("PM_LS_CWALK", -1);
+  const int32_t cw_env = knob("ls_cwalk", -1);
   const bool cluster = cw_env < 0 ? S > 2048 : cw_env != 0;
   const bool use_smem = (cluster ? cwalk_smem_ok(S, optin) : walk_smem_bytes(S) + 1024 <= (size_t)optin) &&
-                        !env_or("PM_LS_SPARSE_GMEM", 0);
+                        !knob("ls_sparse_gmem", 0);
   SpGraph sg;
   {
-    std::lock_guard<std::mutex> lk(g_sp_mu);
     auto key = std::make_tuple(dev, S, st, use_smem, cluster);
     auto it = g_sp_graphs.find(key);
+    if (it == g_sp_graphs.end() && g_sp_graphs.size() >= kSpCacheMax) {
+      PM_CUDA_TRY(cudaDeviceSynchronize());
+      for (auto& kv : g_sp_graphs) {
+        cudaGraphExecDestroy(kv.second.exec);
+        cudaFree(kv.second.dparams);
+      }
+      g_sp_graphs.clear();
+    }
     if (it == g_sp_graphs.end()) {
       SpGraph ng;
       PM_CUDA_TRY(build_sparse_graph(S, use_smem, cluster, ng));

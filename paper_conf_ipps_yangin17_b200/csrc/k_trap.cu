@@ -544,11 +544,6 @@ k_ls_trap(const TrapParams p) {
   }
 }
 
-static int32_t trap_env(const char* name, int32_t dflt) {
-  const char* s = std::getenv(name);
-  return (s && *s) ? (int32_t)std::atoi(s) : dflt;
-}
-
 int32_t ls_trap_min_S() { return 256; }
 
 template <int PPL, int T>
@@ -562,7 +557,7 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   PM_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   const Classes cl(hp.S);
   const int32_t npairs = cl.npairs;
-  int32_t W = trap_env("PM_TRAP_W", X - 2 * T);
+  int32_t W = knob("trap_W", X - 2 * T);
   if (W < T + 1 || W > X - 2 * T) W = X - 2 * T;   // W > T: neighbours publish every halo slot
   hp.W = W;
   hp.nchunks = (npairs + W - 1) / W;
@@ -570,7 +565,7 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   hp.gsz = gsz;
   // cluster mode when every chunk fits one cluster of <= 16 CTAs
   const size_t rep_bytes = sizeof(int32_t) * 4 * (size_t)hp.S;
-  int mode = trap_env("PM_TRAP_CLUSTER", -1);   // -1 auto, 0 grid, 1 cluster
+  int mode = knob("trap_cluster", -1);   // -1 auto, 0 grid, 1 cluster
   int max_cpc_cl = ((size_t)optin > rep_bytes) ? (int)(((size_t)optin - rep_bytes) / SM::bytes) : 0;
   if (max_cpc_cl > 8 / gsz) max_cpc_cl = 8 / gsz;
   // (cluster mode: one chunk per CTA, its neighbours' CTAs = chunks ch +- 1)
@@ -579,9 +574,6 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   // (config 2: 1.50 vs 1.66 ms); with several chunks per CTA the staging of
   // 16 SMs loses to the grid's (config 3: 11.8 vs 10.7 ms)
   if (mode < 0) mode = cl_ok ? 1 : 0;
-  if (trap_env("PM_TRAP_DEBUG", 0))
-    std::fprintf(stderr, "trap: S=%d mode=%d max_cpc_cl=%d nchunks=%d optin=%d bytes=%zu\n", hp.S, mode, max_cpc_cl,
-                 hp.nchunks, optin, SM::bytes);
   if (mode == 1 && !cl_ok) return PM_ERR_UNSUPPORTED;
   if (mode == 1) {
     const int cpc_cl = 1;
@@ -613,11 +605,11 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   }
   // grid mode: cpc chunk groups per CTA, enough CTAs for one pass if possible;
   // neighbour synchronisation (chunk flags, three state buffers) when W >= 2T
-  hp.nbsync = (W >= 2 * T) ? trap_env("PM_TRAP_NBSYNC", 1) : 0;
+  hp.nbsync = (W >= 2 * T) ? knob("trap_nbsync", 1) : 0;
   int max_cpc = (int)((size_t)optin / SM::bytes);
   if (max_cpc > 8 / gsz) max_cpc = 8 / gsz;
   if (max_cpc < 1) return PM_ERR_UNSUPPORTED;
-  int cpc = trap_env("PM_TRAP_CPC", (hp.nchunks + nsm - 1) / nsm);
+  int cpc = knob("trap_cpc", (hp.nchunks + nsm - 1) / nsm);
   if (cpc < 1) cpc = 1;
   if (cpc > max_cpc) cpc = max_cpc;
   const size_t smem = SM::bytes * cpc;
@@ -626,9 +618,6 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
-  if (trap_env("PM_TRAP_DEBUG", 0))
-    std::fprintf(stderr, "trap grid: S=%d W=%d nchunks=%d cpc=%d threads=%d smem=%zu occ=%d\n", hp.S, hp.W,
-                 hp.nchunks, cpc, threads, smem, occ);
   if (occ < 1) return PM_ERR_UNSUPPORTED;
   int grid = (hp.nchunks + cpc - 1) / cpc;
   if (grid > nsm * occ) grid = nsm * occ;
@@ -646,10 +635,11 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   // scratch: 3 round counters, barrier counter, chunk flags [S/2], r1, r2,
   // d0, d1, d2 [S]
   const size_t n = (size_t)S;
-  char* scratch = nullptr;
+  ScopedScratch scr(st), ep(st);
   const size_t head = 64 + sizeof(unsigned int) * (n / 2 + 16);
   const size_t bytes = head + sizeof(int32_t) * 5 * n;
-  PM_CUDA_TRY(pm::scratch_alloc(reinterpret_cast<void**>(&scratch), bytes, st));
+  PM_CUDA_TRY(pm::scratch_alloc(&scr.p, bytes, st));
+  char* scratch = scr.as<char>();
   unsigned long long* rsw = reinterpret_cast<unsigned long long*>(scratch);
   unsigned int* bar = reinterpret_cast<unsigned int*>(scratch + 32);
   unsigned int* flags = reinterpret_cast<unsigned int*>(scratch + 64);
@@ -664,46 +654,40 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.sparse_T = sparse_T; hp.handoff = handoff;
   hp.bar = bar; hp.rsw = rsw;
   hp.out = dev_out; hp.per_round = dev_per_round;
-  hp.prof = trap_env("PM_TRAP_PROF", 0);
+  hp.prof = knob("trap_prof", 0);
   // sigma-permuted rows (the runs become contiguous: 5 instead of 9 16-byte
   // pieces per run at T = 16 from L2, dense sectors instead of stride-2 ones
   // from HBM)
-  int32_t* Ep = nullptr;
   // (measured: config 2 1.25 -> 1.18 ms, config 4 67.4 -> 62.3 ms; config 5
   // 1.09 -> 1.25 s -- building the 16 GiB copy costs more than it saves)
-  const int32_t ep_mode = trap_env("PM_TRAP_EP", 1);   // 0 off, 1 up to E = 2 GiB, 2 always
+  const int32_t ep_mode = knob("trap_ep", 1);   // 0 off, 1 up to E = 2 GiB, 2 always
   if (ep_mode == 2 || ((int64_t)S * ldE * 4 <= (2ll << 30) && ep_mode == 1)) {
     const int32_t m = S - 1, ext = 48;   // >= SPP + 4 for every T used
     const int64_t ldp = ((int64_t)m + ext + 31) / 32 * 32;
-    PM_CUDA_TRY(pm::scratch_alloc(&Ep, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
-    PM_CUDA_TRY(launch_permute_cols(E, ldE, Ep, ldp, S, m, ext, st));
-    hp.Ep = Ep; hp.ldp = ldp;
+    PM_CUDA_TRY(pm::scratch_alloc(&ep.p, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
+    PM_CUDA_TRY(launch_permute_cols(E, ldE, ep.as<int32_t>(), ldp, S, m, ext, st));
+    hp.Ep = ep.as<int32_t>(); hp.ldp = ldp;
   }
   // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
   // used runs win (config 4: 5.0 vs 10.8 us)
-  hp.vec = trap_env("PM_TRAP_VEC", (int64_t)S * ldE * 4 <= (96ll << 20) ? 1 : 0);
-  const int32_t variant = trap_env("PM_TRAP_V", -1);
-  pm_status_t s;
+  hp.vec = knob("trap_vec", (int64_t)S * ldE * 4 <= (96ll << 20) ? 1 : 0);
+  const int32_t variant = knob("trap_variant", -1);
   switch (variant) {
-    case 1: s = launch_trap<1, 8>(hp, st); break;
-    case 2: s = launch_trap<2, 8>(hp, st); break;
-    case 3: s = launch_trap<4, 16>(hp, st); break;
-    case 4: s = launch_trap<4, 8>(hp, st); break;
-    case 5: s = launch_trap<4, 32>(hp, st); break;
+    case 0: return launch_trap<2, 16>(hp, st);
+    case 1: return launch_trap<1, 8>(hp, st);
+    case 2: return launch_trap<2, 8>(hp, st);
+    case 3: return launch_trap<4, 16>(hp, st);
+    case 4: return launch_trap<4, 8>(hp, st);
+    case 5: return launch_trap<4, 32>(hp, st);
     default:
       // measured: 64-pair ranges x 16 classes while E is
       // L2-resident; 128 x 32 from HBM while its 128-thread chunks fit one
       // pass of the grid (config 4: 76.3 -> 67.9 ms; config 5 stays at
       // 64 x 16: 1.21 vs 1.32 s)
-      if ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) s = launch_trap<4, 32>(hp, st);
-      else s = launch_trap<2, 16>(hp, st);
-      break;
+      if ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) return launch_trap<4, 32>(hp, st);
+      return launch_trap<2, 16>(hp, st);
   }
-  if (s != PM_OK) return s;
-  if (Ep) PM_CUDA_TRY(cudaFreeAsync(Ep, st));
-  PM_CUDA_TRY(cudaFreeAsync(scratch, st));
-  return PM_OK;
 }
 
 
@@ -726,7 +710,8 @@ struct TrapRank {                 // one rank's workspace (see trap_ws_layout)
   unsigned int* flags;            // [nchunks] phases completed, per chunk
   unsigned int* bar;              // this rank's grid barrier counter
   unsigned int* xbar;             // cross-rank barrier counter
-  unsigned long long* rtot;       // [3] round swap totals (all ranks add)
+  unsigned long long* rtot;       // [3] round swap totals (all ranks add, system-scope atomics)
+  unsigned int* abort;            // set when a wait timed out (every wait of the launch watches it)
   int32_t* perm;
   const int32_t* E;
   const int32_t* Ep;              // this rank's sigma-permuted copy of E (or NULL)
@@ -739,6 +724,7 @@ struct TrapMultiParams {
   int64_t* per_round;
   int32_t* handoff;               // the first rank's sparse-round flag (or NULL)
   int32_t sparse_T;
+  unsigned long long wait_ns;     // bound of every cross-rank wait
 };
 
 __device__ __forceinline__ int32_t chunk_begin(int32_t r, int32_t nchunks, int32_t world) {
@@ -749,15 +735,62 @@ __device__ __forceinline__ int32_t chunk_owner(int32_t ch, int32_t nchunks, int3
   while (r + 1 < world && chunk_begin(r + 1, nchunks, world) <= ch) ++r;
   return r;
 }
-__device__ __forceinline__ void sys_barrier_arrive_wait(const TrapMultiParams& p, int32_t r, unsigned int target) {
+// Every cross-GPU wait is bounded: a rank that waits longer than the limit
+// (TrapMultiParams::wait_ns, 20 s unless tuned) for a peer sets its
+// workspace's abort flag (and, best effort, every peer's), reports
+// PM_ERR_TIMEOUT and leaves; every other wait of the launch also watches the
+// flag, so no CTA spins forever behind a dead rank.
+
+__device__ __forceinline__ unsigned int ld_acquire_sys(const unsigned int* a) {
+  unsigned int v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys64(const unsigned long long* a) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void raise_abort(const TrapMultiParams& p, int32_t r) {
+  for (int o = 0; o < p.world; ++o)
+    asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(p.rk[o].abort), "r"(1u) : "memory");
+  __threadfence_system();
+  (void)r;
+}
+// wait until *a >= target; false if the launch aborted or the wait timed out
+// (then the abort is raised)
+__device__ __forceinline__ bool wait_ge_sys(const TrapMultiParams& p, int32_t r, const unsigned int* a,
+                                            unsigned int target) {
+  const unsigned long long t0 = gtimer();
+  unsigned int n = 0;
+  while (ld_acquire_sys(a) < target) {
+    if ((++n & 63u) == 0) {
+      if (ld_acquire_sys(p.rk[r].abort)) return false;
+      if (gtimer() - t0 > p.wait_ns) { raise_abort(p, r); return false; }
+    }
+  }
+  return true;
+}
+// the rank's own grid barrier, abortable
+__device__ __forceinline__ bool grid_barrier_mr(const TrapMultiParams& p, int32_t r, unsigned int* bar,
+                                                unsigned int target) {
+  __syncthreads();
+  __shared__ int s_ok;
+  if (threadIdx.x == 0) {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(bar) : "memory");
+    s_ok = wait_ge_sys(p, r, bar, target) ? 1 : 0;
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+  }
+  __syncthreads();
+  return s_ok != 0;
+}
+__device__ __forceinline__ bool sys_barrier_arrive_wait(const TrapMultiParams& p, int32_t r, unsigned int target) {
   // every rank's leader: arrive at every rank's counter, wait for its own
   __threadfence_system();
   for (int o = 0; o < p.world; ++o)
     asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(p.rk[o].xbar) : "memory");
-  unsigned int v;
-  do {
-    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p.rk[r].xbar) : "memory");
-  } while (v < target);
+  return wait_ge_sys(p, r, p.rk[r].xbar, target);
 }
 
 template <int PPL, int T>
@@ -792,20 +825,22 @@ k_ls_trap_mr(const TrapMultiParams p) {
   unsigned int bar_target = 0;
   if (p.out->status != PM_OK) return;   // uniform (written before launch)
 
-  if (threadIdx.x == 0) s_cta_sw = 0;
+  __shared__ int32_t s_abort, s_gab[8];   // s_gab[grp]: written by that group's thread 0 only
+  if (threadIdx.x == 0) { s_cta_sw = 0; s_abort = 0; }
+  if (gt == 0) s_gab[grp] = 0;
   for (int32_t x = lb * blockDim.x + threadIdx.x; x < S; x += nloc * blockDim.x)
     __stcg(me.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(me.rbuf[0] + x) * ld + x));
   bar_target += nloc;
-  grid_barrier(me.bar, bar_target);
+  bool ok = grid_barrier_mr(p, r, me.bar, bar_target);
 
   uint32_t q = 0;
   int32_t rounds = 0;
   int64_t total = 0;
   int status = PM_OK;
   unsigned int xtarget = 0;
-  for (;;) {
+  while (ok) {
     if (leader) me.rtot[(rounds + 1) % 3] = 0ull;
-    for (int32_t c0 = 0; c0 < ncls; c0 += T) {
+    for (int32_t c0 = 0; c0 < ncls && ok; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
       const int32_t u0 = wrap_m(c0 + H, m);
       const int bi = (int)(q % 3u), bn = (int)((q + 1u) % 3u);
@@ -816,13 +851,11 @@ k_ls_trap_mr(const TrapMultiParams p) {
           for (int dch = -1; dch <= 1; dch += 2) {
             const int32_t c2 = ch + dch;
             if (c2 < 0 || c2 >= nch) continue;
-            unsigned int v;
-            do {
-              asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(me.flags + c2) : "memory");
-            } while (v < q);
+            if (!wait_ge_sys(p, r, me.flags + c2, q)) { s_gab[grp] = 1; s_abort = 1; break; }
           }
         }
         group_sync(1 + grp, GT);
+        if (s_gab[grp]) break;   // group-uniform: written by this group's thread 0 before the sync
         if (have) {
           TrapChunk C;
           const int32_t k0 = ch * W, k1 = min(k0 + W, K + 1);
@@ -882,24 +915,28 @@ k_ls_trap_mr(const TrapMultiParams p) {
       if ((threadIdx.x & 31) == 0 && mysw) atomicAdd(&s_cta_sw, mysw);
       ++q;
       __syncthreads();
+      if (s_abort) { ok = false; break; }
       if (c0 + T >= ncls) {
-        // round end: every CTA's count to every rank's total, then the rank
-        // barrier and the cross-rank barrier, then the rank barrier again
+        // round end: every CTA's count to every rank's total (system-scope
+        // atomics: the adds of several GPUs meet in one counter), then the
+        // rank barrier and the cross-rank barrier, then the rank barrier again
         if (threadIdx.x == 0 && s_cta_sw) {
-          for (int o = 0; o < world; ++o) atomicAdd(p.rk[o].rtot + rounds % 3, (unsigned long long)s_cta_sw);
+          for (int o = 0; o < world; ++o)
+            atomicAdd_system(p.rk[o].rtot + rounds % 3, (unsigned long long)s_cta_sw);
         }
         if (threadIdx.x == 0) s_cta_sw = 0;
         bar_target += nloc;
-        grid_barrier(me.bar, bar_target);
+        if (!grid_barrier_mr(p, r, me.bar, bar_target)) { ok = false; break; }
         if (leader) {
           xtarget += (unsigned)world;
-          sys_barrier_arrive_wait(p, r, xtarget);
+          if (!sys_barrier_arrive_wait(p, r, xtarget)) s_abort = 1;
         }
         bar_target += nloc;
-        grid_barrier(me.bar, bar_target);
+        if (!grid_barrier_mr(p, r, me.bar, bar_target) || s_abort) { ok = false; break; }
       }
     }
-    if (threadIdx.x == 0) s_rs = *((volatile unsigned long long*)(me.rtot + rounds % 3));
+    if (!ok) break;
+    if (threadIdx.x == 0) s_rs = ld_acquire_sys64(me.rtot + rounds % 3);
     __syncthreads();
     const int64_t rs = (int64_t)s_rs;
     if (leader && r == p.rank0 && rounds < p.max_log) p.per_round[rounds] = rs;
@@ -912,6 +949,15 @@ k_ls_trap_mr(const TrapMultiParams p) {
       if (leader && r == p.rank0) *p.handoff = 1;
       break;
     }
+  }
+  if (!ok) {   // a peer did not arrive in time: report and leave (nothing is written to perm)
+    if (leader && r == p.rank0) {
+      p.out->status = PM_ERR_TIMEOUT;
+      p.out->rounds = rounds;
+      p.out->swaps = total;
+      if (p.handoff) *p.handoff = 0;
+    }
+    return;
   }
   // every chunk's owned slots (class ncls - 1) into every rank's perm
   const int32_t* fin = me.rbuf[q % 3u];
@@ -928,12 +974,12 @@ k_ls_trap_mr(const TrapMultiParams p) {
     }
   }
   bar_target += nloc;
-  grid_barrier(me.bar, bar_target);
+  ok = grid_barrier_mr(p, r, me.bar, bar_target);
   if (leader) {
     xtarget += (unsigned)world;
-    sys_barrier_arrive_wait(p, r, xtarget);
+    if (ok) ok = sys_barrier_arrive_wait(p, r, xtarget);
     if (r == p.rank0) {
-      p.out->status = status;
+      p.out->status = ok ? status : PM_ERR_TIMEOUT;
       p.out->rounds = rounds;
       p.out->swaps = total;
     }
@@ -952,6 +998,7 @@ static void trap_ws_layout(void* ws, int32_t S, int32_t* perm, const int32_t* E,
   rk.rtot = reinterpret_cast<unsigned long long*>(b);
   rk.bar = reinterpret_cast<unsigned int*>(b + 32);
   rk.xbar = reinterpret_cast<unsigned int*>(b + 64);
+  rk.abort = reinterpret_cast<unsigned int*>(b + 96);
   rk.flags = reinterpret_cast<unsigned int*>(b + 128);
   int32_t* base = reinterpret_cast<int32_t*>(b + 128 + sizeof(unsigned int) * (n / 2 + 16));
   rk.rbuf[0] = perm; rk.rbuf[1] = base; rk.rbuf[2] = base + n;
@@ -985,6 +1032,7 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.handoff = handoff; hp.sparse_T = sparse_T;
   hp.ldp = ldp;
+  hp.wait_ns = (unsigned long long)knob("trap_wait_ms", 20000) * 1000000ull;
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
   int max_cpc = (int)((size_t)optin / SM::bytes);
@@ -1008,14 +1056,17 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   return PM_OK;
 }
 
+static int32_t trap_multi_variant(int32_t S, int64_t ldE) {
+  int32_t v = knob("trap_variant", -1);
+  if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) ? 5 : 0;
+  return v;
+}
 // Chunk geometry as the single-GPU grid mode: 64 x 16 while E is
 // L2-resident or S > 16384, else 128 x 32 (PM_TRAP_V = 0 / 5 force one).
 pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
                            int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                            cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0, int64_t ldp = 0) {
-  int32_t v = trap_env("PM_TRAP_V", -1);
-  if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) ? 5 : 0;
-  if (v == 5)
+  if (trap_multi_variant(S, ldE) == 5)
     return launch_trap_multi<4, 32>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
                                     st, handoff, sparse_T, ldp);
   return launch_trap_multi<2, 16>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
@@ -1028,7 +1079,7 @@ static pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaS
                                  int64_t* ldp) {
   *Ep = nullptr;
   *ldp = 0;
-  const int32_t ep_mode = trap_env("PM_TRAP_EP", 1);
+  const int32_t ep_mode = knob("trap_ep", 1);
   if (ep_mode == 0 || (ep_mode == 1 && (int64_t)S * ldE * 4 > (2ll << 30))) return PM_OK;
   const int32_t m = S - 1, ext = 48;
   *ldp = ((int64_t)m + ext + 31) / 32 * 32;
@@ -1037,16 +1088,30 @@ static pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaS
   return PM_OK;
 }
 
+// Can the multi-rank kernel take (S, world)?  Checked before anything is
+// enqueued (pm.h: arguments are validated before any launch).
+pm_status_t trap_multi_supported(int32_t S, int64_t ldE, int32_t world) {
+  if (world < 1 || world > kMaxRanks) return PM_ERR_INVALID;
+  if (S < ls_trap_min_S() || (S & 1)) return PM_ERR_UNSUPPORTED;
+  const int32_t W = trap_multi_variant(S, ldE) == 5 ? 64 : 32;   // X - 2T of the geometry
+  if ((Classes(S).npairs + W - 1) / W < world) return PM_ERR_UNSUPPORTED;
+  return PM_OK;
+}
+
 // All ranks of a world on the current device, one launch (test hook).
 pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
                                 int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                                 cudaStream_t st) {
-  if (world < 1 || world > kMaxRanks) return PM_ERR_UNSUPPORTED;
+  {
+    const pm_status_t v = trap_multi_supported(S, ldE, world);
+    if (v != PM_OK) return v;
+  }
   PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
   const size_t wsb = (trap_ws_bytes(S) + 255) / 256 * 256;
   const size_t pb = ((size_t)S * sizeof(int32_t) + 255) / 256 * 256;
-  char* buf = nullptr;
-  PM_CUDA_TRY(pm::scratch_alloc(reinterpret_cast<void**>(&buf), (wsb + pb) * world, st));
+  ScopedScratch bufs(st), sps(st), ep(st);
+  PM_CUDA_TRY(pm::scratch_alloc(&bufs.p, (wsb + pb) * world, st));
+  char* buf = bufs.as<char>();
   TrapRank ranks[kMaxRanks];
   for (int r = 0; r < world; ++r) {
     char* ws = buf + (wsb + pb) * r;
@@ -1063,24 +1128,25 @@ pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_
     const pm_status_t s0 = sparse_prepare(E, ldE, S, ranks[world - 1].perm, max_rounds, dev_out, dev_per_round,
                                           max_log, st, &sr);
     if (s0 != PM_OK) return s0;
+    sps.p = sr.scratch;   // freed here on an error path; sparse_launch frees it otherwise
   }
-  int32_t* Ep = nullptr;
   int64_t ldp = 0;
   {
+    int32_t* Ep = nullptr;
     const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+    ep.p = Ep;
     if (se != PM_OK) return se;
   }
-  for (int r = 0; r < world; ++r) ranks[r].Ep = Ep;
+  for (int r = 0; r < world; ++r) ranks[r].Ep = ep.as<int32_t>();
   pm_status_t s = run_trap_multi(ranks, world, 0, world, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
                                  sr.pending, sparse_T, ldp);
   if (s != PM_OK) return s;
-  if (Ep) PM_CUDA_TRY(cudaFreeAsync(Ep, st));
   if (sparse_T > 0) {
+    sps.p = nullptr;
     const pm_status_t s1 = sparse_launch(&sr, st);
     if (s1 != PM_OK) return s1;
   }
   PM_CUDA_TRY(cudaMemcpyAsync(perm, ranks[world - 1].perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
-  PM_CUDA_TRY(cudaFreeAsync(buf, st));
   return PM_OK;
 }
 
@@ -1091,30 +1157,42 @@ pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_
 pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* const* perm_peers,
                             void* const* ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
                             LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st) {
-  if (world < 1 || world > kMaxRanks || rank < 0 || rank >= world) return PM_ERR_INVALID;
+  if (rank < 0 || rank >= world) return PM_ERR_INVALID;
+  {
+    const pm_status_t v = trap_multi_supported(S, ldE, world);
+    if (v != PM_OK) return v;
+  }
+  // a non-bijection would send out-of-range tile indices into E; every rank
+  // holds the same perm, so every rank's kernel returns at once (status set)
+  PM_CUDA_TRY(launch_perm_check(perm_peers[rank], S, dev_out, st));
   TrapRank ranks[kMaxRanks];
   for (int r = 0; r < world; ++r) trap_ws_layout(ws_peers[r], S, perm_peers[r], E, ranks[r]);
   // quiet rounds: this rank continues alone (sparse rounds on its own copy
   // of r and E -- every rank reaches the same result, no exchange)
   const int32_t sparse_T = ls_sparse_threshold(S, PM_LS_TRAP);
+  ScopedScratch sps(st), ep(st);
   SparseRun sr;
   if (sparse_T > 0) {
     const pm_status_t s0 = sparse_prepare(E, ldE, S, perm_peers[rank], max_rounds, dev_out, dev_per_round, max_log,
                                           st, &sr);
     if (s0 != PM_OK) return s0;
+    sps.p = sr.scratch;
   }
-  int32_t* Ep = nullptr;
   int64_t ldp = 0;
   {
+    int32_t* Ep = nullptr;
     const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+    ep.p = Ep;
     if (se != PM_OK) return se;
   }
-  ranks[rank].Ep = Ep;   // only this rank's entry is read by this launch
+  ranks[rank].Ep = ep.as<int32_t>();   // only this rank's entry is read by this launch
   const pm_status_t s = run_trap_multi(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
                                        st, sr.pending, sparse_T, ldp);
   if (s != PM_OK) return s;
-  if (Ep) PM_CUDA_TRY(cudaFreeAsync(Ep, st));
-  if (sparse_T > 0) return sparse_launch(&sr, st);
+  if (sparse_T > 0) {
+    sps.p = nullptr;
+    return sparse_launch(&sr, st);
+  }
   return PM_OK;
 }
 }  // namespace pm

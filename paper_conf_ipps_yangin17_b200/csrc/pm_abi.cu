@@ -8,33 +8,67 @@
 
 #include "pm_internal.cuh"
 
+#include <cstring>
+#include <map>
 #include <mutex>
+#include <string>
 
 namespace pm {
 std::atomic<int64_t> g_launches{0};
 
+// ---- scratch pool ----------------------------------------------------------
+static std::mutex g_pool_mu;
+static cudaMemPool_t g_pools[64] = {};
+
 cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
-  static std::mutex mu;
-  static cudaMemPool_t pools[64] = {};
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   cudaMemPool_t pool;
   {
-    std::lock_guard<std::mutex> lk(mu);
-    if (!pools[dev]) {
+    std::lock_guard<std::mutex> lk(g_pool_mu);
+    if (!g_pools[dev]) {
       cudaMemPoolProps props = {};
       props.allocType = cudaMemAllocationTypePinned;
       props.location.type = cudaMemLocationTypeDevice;
       props.location.id = dev;
-      if ((e = cudaMemPoolCreate(&pools[dev], &props)) != cudaSuccess) return e;
-      uint64_t thr = UINT64_MAX;
-      if ((e = cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &thr)) != cudaSuccess) return e;
+      if ((e = cudaMemPoolCreate(&g_pools[dev], &props)) != cudaSuccess) return e;
+      // keep up to kPoolKeepBytes mapped between calls (the per-call scratch of
+      // configs 1-4 is served without re-mapping); anything beyond goes back to
+      // the driver at the next synchronisation (pm.h "Ownership")
+      uint64_t thr = kPoolKeepBytes;
+      if ((e = cudaMemPoolSetAttribute(g_pools[dev], cudaMemPoolAttrReleaseThreshold, &thr)) != cudaSuccess)
+        return e;
     }
-    pool = pools[dev];
+    pool = g_pools[dev];
   }
   return cudaMallocFromPoolAsync(p, bytes, pool, st);
+}
+
+// ---- tuning overrides (tests / development; never read from the environment)
+static std::mutex g_tune_mu;
+static std::map<std::string, int32_t> g_tune;
+
+static const char* const kTuningNames[] = {
+    "trap_variant", "trap_W", "trap_cluster", "trap_nbsync", "trap_cpc", "trap_prof", "trap_ep", "trap_vec",
+    "trap_spec",    "trap_prefetch", "trap_wait_ms",
+    "ls_sparse",    "ls_sparse_T", "ls_cwalk", "ls_sparse_gmem",
+    "auction_gs",   "auction_keep", "auction_smem_price", "auction_theta", "auction_eps_shift",
+    "auction_max_rounds", "auction_ctas_per_sm"};
+
+bool tuning_name_ok(const char* name) {
+  if (!name) return false;
+  for (const char* n : kTuningNames)
+    if (std::strcmp(n, name) == 0) return true;
+  return false;
+}
+
+int32_t knob(const char* name, int32_t dflt) {
+  std::lock_guard<std::mutex> lk(g_tune_mu);
+  if (g_tune.empty()) return dflt;
+  auto it = g_tune.find(name);
+  return it == g_tune.end() ? dflt : it->second;
 }
 
 static std::mutex g_ctr_mu;
@@ -92,10 +126,16 @@ struct DevBuf {
   ~DevBuf() { if (p) cudaFreeAsync(p, st); }
 };
 
+// PM_LS_* values 2 and 4 were retired in round 2 (dominated methods)
+bool valid_method(int32_t method) {
+  return method == PM_LS_AUTO || method == PM_LS_CLASS || method == PM_LS_WINDOW || method == PM_LS_WALK ||
+         method == PM_LS_TRAP;
+}
+
 bool valid_ls_args(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm, int32_t max_rounds,
                    int32_t method) {
   if (!d_E || !d_perm || S < 1 || ld_E < S || max_rounds < 0) return false;
-  return method >= PM_LS_AUTO && method <= PM_LS_TRAP;
+  return valid_method(method);
 }
 
 // Synchronous local search: scratch, launch, read back.
@@ -140,6 +180,7 @@ const char* pm_status_string(pm_status_t s) {
     case PM_ERR_NOT_CONVERGED: return "PM_ERR_NOT_CONVERGED: max_rounds reached before a zero-swap round";
     case PM_ERR_UNSUPPORTED: return "PM_ERR_UNSUPPORTED: not supported by this build/device";
     case PM_ERR_NOT_PERMUTATION: return "PM_ERR_NOT_PERMUTATION: perm is not a bijection of [0, S)";
+    case PM_ERR_TIMEOUT: return "PM_ERR_TIMEOUT: a peer rank did not arrive in time";
   }
   return "PM_ERR_?: unknown status";
 }
@@ -242,6 +283,10 @@ pm_status_t pm_local_search_ex(const int32_t* d_E, int64_t ld_E, int32_t S, int3
 pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
                                   int32_t max_rounds, int32_t method, int64_t* d_result, pm_stream_t stream) {
   if (!d_result || !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method)) return PM_ERR_INVALID;
+  {
+    const pm_status_t v = ls_method_supported(S, method);
+    if (v != PM_OK) return v;
+  }
   cudaStream_t st = (cudaStream_t)stream;
   PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
   int32_t used = method;
@@ -264,6 +309,10 @@ pm_status_t pm_local_search_multi_async(const int32_t* d_E, int64_t ld_E, int32_
   if (world < 1 || rank < 0 || rank >= world) return PM_ERR_INVALID;
   for (int r = 0; r < world; ++r)
     if (!d_perm_peers[r] || !d_ws_peers[r]) return PM_ERR_INVALID;
+  {
+    const pm_status_t v = trap_multi_supported(S, ld_E, world);
+    if (v != PM_OK) return v;
+  }
   cudaStream_t st = (cudaStream_t)stream;
   PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
   return trap_multi_rank(d_E, ld_E, S, d_perm_peers, d_ws_peers, rank, world, max_rounds,
@@ -274,6 +323,10 @@ pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int
                                            int32_t world, int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
                                            pm_stream_t stream) {
   if (!d_E || !d_perm || ld_E < S || max_rounds < 0 || world < 1) return PM_ERR_INVALID;
+  {
+    const pm_status_t v = trap_multi_supported(S, ld_E, world);
+    if (v != PM_OK) return v;
+  }
   cudaStream_t st = (cudaStream_t)stream;
   DevBuf buf;
   buf.st = st;
@@ -289,8 +342,6 @@ pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int
   if (h_swaps) *h_swaps = h.swaps;
   return (pm_status_t)h.status;
 }
-
-int32_t pm_ls_cta_max_S(void) { return ls_cta_max_S(); }
 
 int32_t pm_ls_auto_method(int32_t S) {
   // measured on B200 (whole search incl. sparse rounds): TRAP for
@@ -332,10 +383,14 @@ pm_status_t pm_photomosaic_async(const uint8_t* d_input, const uint8_t* d_target
                                  int32_t* d_E, int64_t ld_E, int32_t* d_perm, int32_t method, int64_t* d_result,
                                  pm_stream_t stream) {
   if (!d_input || !d_target || !d_E || !d_perm || !d_result || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
-  if (method < PM_LS_AUTO || method > PM_LS_TRAP) return PM_ERR_INVALID;
+  if (!valid_method(method)) return PM_ERR_INVALID;
   const int32_t g = N / M;
   const int32_t S = g * g;
   if (ld_E < S) return PM_ERR_INVALID;
+  {
+    const pm_status_t v = ls_method_supported(S, method);   // before Steps 1-2 are enqueued
+    if (v != PM_OK) return v;
+  }
   cudaStream_t st = (cudaStream_t)stream;
   pm_status_t s = pm_error_matrix(d_input, d_target, N, M, C, 0, S, d_E, ld_E, stream);   // Steps 1-2
   if (s != PM_OK) return s;
@@ -369,10 +424,15 @@ pm_status_t pm_photomosaic(const uint8_t* d_input, const uint8_t* d_target, int3
 pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target, int32_t N, int32_t M, int32_t C,
                                 int32_t method, int32_t* h_perm, int32_t* h_rounds, int64_t* h_swaps,
                                 int64_t* h_cost, pm_stream_t stream) {
-  if (!h_input || !h_target || !h_perm || !valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  if (!h_input || !h_target || !h_perm || !valid_image_args(N, M, C) || !valid_method(method))
+    return PM_ERR_INVALID;
   cudaStream_t st = (cudaStream_t)stream;
   const int32_t g = N / M;
   const int64_t S = (int64_t)g * g;
+  {
+    const pm_status_t v = ls_method_supported((int32_t)S, method);
+    if (v != PM_OK) return v;
+  }
   const size_t img = (size_t)N * N * C;
   const size_t bytes = 64 + 2 * img + sizeof(int32_t) * (size_t)S * (size_t)S + sizeof(int32_t) * (size_t)S + 64;
   DevBuf buf;
@@ -426,5 +486,36 @@ pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, i
 }
 
 int64_t pm_launch_count(void) { return g_launches.load() + device_launch_total(); }
+
+pm_status_t pm_tuning_set(const char* name, int32_t value) {
+  if (!tuning_name_ok(name)) return PM_ERR_INVALID;
+  std::lock_guard<std::mutex> lk(g_tune_mu);
+  g_tune[name] = value;
+  return PM_OK;
+}
+
+void pm_tuning_reset(void) {
+  std::lock_guard<std::mutex> lk(g_tune_mu);
+  g_tune.clear();
+}
+
+pm_status_t pm_scratch_trim(void) {
+  int dev = 0;
+  PM_CUDA_TRY(cudaGetDevice(&dev));
+  if (dev < 0 || dev >= 64) return PM_ERR_CUDA;
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (g_pools[dev]) PM_CUDA_TRY(cudaMemPoolTrimTo(g_pools[dev], 0));
+  return PM_OK;
+}
+
+size_t pm_scratch_reserved_bytes(void) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (!g_pools[dev]) return 0;
+  uint64_t v = 0;
+  if (cudaMemPoolGetAttribute(g_pools[dev], cudaMemPoolAttrReservedMemCurrent, &v) != cudaSuccess) return 0;
+  return (size_t)v;
+}
 
 }  // extern "C"

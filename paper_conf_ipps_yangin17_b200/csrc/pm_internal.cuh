@@ -15,15 +15,33 @@ namespace pm {
 extern std::atomic<int64_t> g_launches;
 inline void note_launch(int64_t n = 1) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
-// Stream-ordered scratch from a library-owned memory pool per device whose
-// release threshold is unlimited: after the first call, scratch allocations
-// are served from the pool without re-mapping memory (the default pool
-// returns memory to the driver at every synchronisation, ~1 ms per call).
+// Stream-ordered scratch from a library-owned memory pool per device that keeps
+// up to kPoolKeepBytes mapped between calls: the scratch of repeated calls is
+// served without re-mapping (the default pool returns memory to the driver at
+// every synchronisation, ~1 ms per call); pm_scratch_trim() releases it all.
 cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st);
+constexpr uint64_t kPoolKeepBytes = 4ull << 30;   // pool release threshold
 template <typename T>
 inline cudaError_t scratch_alloc(T** p, size_t bytes, cudaStream_t st) {
   return scratch_alloc(reinterpret_cast<void**>(p), bytes, st);
 }
+
+// Tuning overrides (pm_tuning_set): the measured defaults unless a test or a
+// development tool overrode them through the ABI.  Never read from the
+// environment; every override keeps results bit-exact.
+int32_t knob(const char* name, int32_t dflt);
+bool tuning_name_ok(const char* name);
+
+// Scratch owned by a scope: freed (stream-ordered) on every return path.
+struct ScopedScratch {
+  void* p = nullptr;
+  cudaStream_t st = nullptr;
+  explicit ScopedScratch(cudaStream_t s) : st(s) {}
+  ScopedScratch(const ScopedScratch&) = delete;
+  ScopedScratch& operator=(const ScopedScratch&) = delete;
+  ~ScopedScratch() { if (p) cudaFreeAsync(p, st); }
+  template <typename T> T* as() const { return static_cast<T*>(p); }
+};
 
 #define PM_CUDA_TRY(expr)                         \
   do {                                            \
@@ -101,7 +119,6 @@ struct LsResult {
   int64_t swaps;
 };
 cudaError_t launch_iota(int32_t* perm, int32_t S, cudaStream_t st);
-int32_t ls_cta_max_S();
 // Runs the whole search; writes device results (LsResult + per-round swaps)
 // into dev_out (LsResult) and dev_per_round (int64 [max_log]).
 pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm,
@@ -110,13 +127,9 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
                              int32_t* used_method);
 int32_t ls_class_launches_per_round(int32_t S);
 int32_t ls_window_max_S();
-int32_t ls_pairwin_min_S();
-int32_t ls_pairwin_max_S();
 // Ep[t][pos] = E[t][2 pos mod m], pos in [0, m + ext) (sigma-permuted rows, k_window.cu)
 cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int64_t ldp, int32_t S, int32_t m,
                                 int32_t ext, cudaStream_t st);
-pm_status_t run_pairwin(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
-                        LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                        LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
                        int32_t* handoff = nullptr, int32_t sparse_T = 0);
@@ -176,6 +189,9 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
 // Multi-rank TRAP (k_trap.cu).
 struct TrapRank;
 size_t trap_ws_bytes(int32_t S);
+pm_status_t trap_multi_supported(int32_t S, int64_t ldE, int32_t world);
+// PM_OK if `method` (resolved: not AUTO) runs at this S, else PM_ERR_UNSUPPORTED
+pm_status_t ls_method_supported(int32_t S, int32_t method);
 size_t trap_ws_zero_bytes(int32_t S);
 pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
                                 int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,

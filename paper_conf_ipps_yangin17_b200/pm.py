@@ -19,8 +19,9 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libpm.so")
 
-PM_OK, PM_ERR_INVALID, PM_ERR_CUDA, PM_ERR_NOT_CONVERGED, PM_ERR_UNSUPPORTED, PM_ERR_NOT_PERMUTATION = range(6)
-METHODS = {"auto": 0, "class": 1, "cta": 2, "window": 3, "pairwin": 4, "walk": 5, "trap": 6}
+(PM_OK, PM_ERR_INVALID, PM_ERR_CUDA, PM_ERR_NOT_CONVERGED, PM_ERR_UNSUPPORTED, PM_ERR_NOT_PERMUTATION,
+ PM_ERR_TIMEOUT) = range(7)
+METHODS = {"auto": 0, "class": 1, "window": 3, "walk": 5, "trap": 6}
 
 _lib = None
 _P = ctypes.c_void_p
@@ -38,7 +39,6 @@ _SIGS = [
     ("pm_local_search", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _P, _P, _P]),
     ("pm_local_search_ex", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P, _I32, _P]),
     ("pm_local_search_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P]),
-    ("pm_ls_cta_max_S", _I32, []),
     ("pm_ls_auto_method", _I32, [_I32]),
     ("pm_init_identity", ctypes.c_int, [_P, _I32, _P]),
     ("pm_cost", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P]),
@@ -53,6 +53,10 @@ _SIGS = [
     ("pm_trap_workspace_reset", ctypes.c_int, [_P, _I32, _P]),
     ("pm_local_search_multi_async", ctypes.c_int, [_P, _I64, _I32, _P, _P, _I32, _I32, _I32, _P, _P]),
     ("pm_local_search_multi_emulated", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P]),
+    ("pm_tuning_set", ctypes.c_int, [ctypes.c_char_p, _I32]),
+    ("pm_tuning_reset", None, []),
+    ("pm_scratch_trim", ctypes.c_int, []),
+    ("pm_scratch_reserved_bytes", ctypes.c_size_t, []),
 ]
 
 
@@ -247,10 +251,6 @@ def local_search_multi_async(E, perm_ptrs, ws_ptrs, rank: int, world: int, resul
            "pm_local_search_multi_async")
 
 
-def ls_cta_max_S() -> int:
-    return int(lib().pm_ls_cta_max_S())
-
-
 def ls_auto_method(S: int) -> str:
     """Name of the method PM_LS_AUTO picks for S on the current device."""
     code = int(lib().pm_ls_auto_method(S))
@@ -357,3 +357,37 @@ def optimal_assignment(E, perm=None, price=None, stream=None):
 
 def launch_count() -> int:
     return int(lib().pm_launch_count())
+
+
+# ------------------------------------------------ tuning / scratch (pm.h) ---
+def tuning_set(name: str, value: int):
+    """pm_tuning_set: override one measured default (tests / dev tools)."""
+    _check(lib().pm_tuning_set(name.encode(), int(value)), f"pm_tuning_set({name})")
+
+
+def tuning_reset():
+    lib().pm_tuning_reset()
+
+
+class tuning:
+    """Context manager: ``with pm.tuning(trap_variant=3, ls_sparse=0): ...``
+    (every override is dropped on exit)."""
+
+    def __init__(self, **knobs):
+        self.knobs = knobs
+
+    def __enter__(self):
+        for k, v in self.knobs.items():
+            tuning_set(k, v)
+        return self
+
+    def __exit__(self, *exc):
+        tuning_reset()
+
+
+def scratch_trim():
+    _check(lib().pm_scratch_trim(), "pm_scratch_trim")
+
+
+def scratch_reserved_bytes() -> int:
+    return int(lib().pm_scratch_reserved_bytes())

@@ -52,8 +52,37 @@ def test_library_is_sm100a(pm):
 
 
 def test_status_strings(pm):
-    for s in range(6):
+    for s in range(7):
         assert pm.status_string(s).startswith("PM_")
+    assert "TIMEOUT" in pm.status_string(pm.PM_ERR_TIMEOUT)
+
+
+def test_tuning_overrides_are_explicit(pm):
+    # development overrides go through the ABI only (never the environment):
+    # unknown names are rejected, known ones accepted, reset restores defaults
+    L = pm.lib()
+    assert L.pm_tuning_set(b"no_such_knob", 1) == pm.PM_ERR_INVALID
+    assert L.pm_tuning_set(None, 1) == pm.PM_ERR_INVALID
+    for name in ("trap_variant", "trap_cluster", "ls_sparse_T", "ls_cwalk", "auction_gs"):
+        assert L.pm_tuning_set(name.encode(), 1) == pm.PM_OK
+    pm.tuning_reset()
+    with pytest.raises(pm.PMError):
+        pm.tuning_set("PM_TRAP_V", 3)      # the round-1 environment names are gone
+
+
+def test_release_library_reads_no_environment():
+    # the library's own sources never read the environment: behaviour cannot
+    # depend on the caller's environment (tuning overrides are explicit ABI
+    # calls; the static CUDA runtime still reads its own CUDA_* variables)
+    csrc = os.path.join(ROOT, "paper_conf_ipps_yangin17_b200", "csrc")
+    for f in os.listdir(csrc):
+        src = open(os.path.join(csrc, f)).read()
+        assert "getenv(" not in src and "std::getenv" not in src, f
+
+
+def test_retired_methods_rejected(pm):
+    # PM_LS_* 2 and 4 (round-1 single-CTA / pair-window methods) are retired
+    assert set(pm.METHODS.values()) == {0, 1, 3, 5, 6}
 
 
 def test_tile_stride(pm):

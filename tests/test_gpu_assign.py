@@ -121,15 +121,16 @@ def test_assignment_rejects_out_of_range_weights():
 @pytest.mark.parametrize("gs", ["0", "1", "256"])
 @pytest.mark.parametrize("knobs", [("8", "3"), ("2", "0"), ("64", "20")])
 @pytest.mark.parametrize("keep,smem", [("0", "1"), ("1", "0")])
-def test_assignment_schedule_knobs_stay_exact(monkeypatch, gs, knobs, keep, smem):
+def test_assignment_schedule_knobs_stay_exact(gs, knobs, keep, smem):
     """Exactness does not depend on the eps schedule, on where the
     Gauss-Seidel tail takes over, on keeping eps-CS pairs across phases or on
     where the tail keeps its prices (any eps0 >= 1, any divisor, final eps = 1)."""
-    monkeypatch.setenv("PM_AUCTION_GS", gs)
-    monkeypatch.setenv("PM_AUCTION_KEEP", keep)
-    monkeypatch.setenv("PM_AUCTION_SMEM_PRICE", smem)
-    monkeypatch.setenv("PM_AUCTION_THETA", knobs[0])
-    monkeypatch.setenv("PM_AUCTION_EPS_SHIFT", knobs[1])
+    with pm.tuning(auction_gs=int(gs), auction_keep=int(keep), auction_smem_price=int(smem),
+                   auction_theta=int(knobs[0]), auction_eps_shift=int(knobs[1])):
+        _schedule_case()
+
+
+def _schedule_case():
     rng = np.random.default_rng(77)
     for S in (5, 64, 130):
         E = rng.integers(0, 2000, size=(S, S)).astype(np.int32)

@@ -24,6 +24,14 @@ DEV = torch.device("cuda:0")
 _cache = {}
 
 
+@pytest.fixture(autouse=True)
+def _reset_tuning():
+    # overrides set by a test (pm.tuning_set) never leak into the next one
+    pm.tuning_reset()
+    yield
+    pm.tuning_reset()
+
+
 def pair(fam, N, M, C=3, seed=0):
     key = ("img", fam, N, M, C, seed)
     if key not in _cache:
@@ -134,8 +142,7 @@ def test_error_matrix_config5_row_chunks_sampled():
 
 # ------------------------------------------------------------------ Alg. 2 --
 def _supported(method, S):
-    return (not (method == "pairwin" and not (40 <= S <= 2048)) and not (method == "window" and S > 2048)
-            and not (method == "trap" and (S < 256 or S % 2)))
+    return not (method == "window" and S > 2048) and not (method == "trap" and (S < 256 or S % 2))
 
 
 def _check_ls(E_np, method, perm0=None, max_rounds=0):
@@ -153,39 +160,39 @@ def _check_ls(E_np, method, perm0=None, max_rounds=0):
     return ref
 
 
-@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "window", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "shuffle", "transposition", "identical"])
 def test_local_search_parity_config1(method, fam):
     _check_ls(oracle_E(fam, 128, 8), method)
 
 
-@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "window", "class"])
 @pytest.mark.parametrize("fam", ["smooth", "noise", "ties"])
 def test_local_search_parity_config2(method, fam):
     _check_ls(oracle_E(fam, 512, 16), method)
 
 
-@pytest.mark.parametrize("method", ["auto", "trap", "walk", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "trap", "walk", "class"])
 def test_local_search_parity_config3(method):
     ref = _check_ls(oracle_E("smooth", 1024, 16), method)
     assert ref[1] >= 3
 
 
-@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "window", "class"])
 @pytest.mark.parametrize("N,M,C", [(90, 10, 3), (42, 6, 3), (200, 5, 1), (48, 16, 3), (30, 10, 3), (64, 64, 1)])
 def test_local_search_parity_ragged_and_odd(method, N, M, C):
     # S = 81, 49, 9 are odd (the fixed point idles, reading R9); S = 1 trivial
     _check_ls(oracle_E("smooth", N, M, C), method)
 
 
-@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "window", "class"])
 def test_local_search_resume_from_any_bijection(method):
     E = oracle_E("noise", 128, 8)
     rng = np.random.default_rng(3)
     _check_ls(E, method, perm0=rng.permutation(256).astype(np.int32))
 
 
-@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "window", "class"])
 def test_local_search_max_rounds_then_resume(method):
     E_np = oracle_E("smooth", 512, 16)
     ref = _check_ls(E_np, method, max_rounds=2)
@@ -193,7 +200,7 @@ def test_local_search_max_rounds_then_resume(method):
     _check_ls(E_np, method, perm0=ref[0])
 
 
-@pytest.mark.parametrize("method", ["trap", "walk", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["trap", "walk", "window", "class"])
 def test_local_search_rejects_non_permutation(method):
     E = dev(oracle_E("smooth", 128, 8))
     bad = torch.arange(256, dtype=torch.int32, device=DEV)
@@ -208,15 +215,26 @@ def test_local_search_rejects_non_permutation(method):
 
 
 def test_local_search_random_small_matrices():
-    # tie-heavy random E for S <= 9 against the oracle replay, both methods
+    # tie-heavy random E for S <= 9 against the oracle replay, every method
+    # that takes such S
     rng = np.random.default_rng(0)
     for _ in range(25):
         S = int(rng.integers(1, 10))
         E = rng.integers(0, 4, size=(S, S)).astype(np.int32)
-        for method in ("walk", "window", "cta", "class"):
+        for method in ("walk", "window", "class"):
             _check_ls(E, method)
-        if S >= 40:
-            _check_ls(E, "pairwin")
+
+
+@pytest.mark.parametrize("S", [256, 258, 300, 512])
+@pytest.mark.parametrize("hi", [2, 4, 50])
+def test_trap_tie_heavy_random_E(S, hi):
+    # TRAP's smallest S with random E whose entries take only `hi` values:
+    # many line-5 ties (strict '>', reading R6), swaps anywhere incl. pair 0
+    rng = np.random.default_rng(S * 100 + hi)
+    E = rng.integers(0, hi, size=(S, S)).astype(np.int32)
+    _check_ls(E, "trap")
+    with pm.tuning(ls_sparse=0):
+        _check_ls(E, "trap")
 
 
 def _two_opt_gpu(E, perm):
@@ -295,7 +313,7 @@ def test_cost_int64():
 
 
 # -------------------------------------------------------------- pipeline ----
-@pytest.mark.parametrize("method", ["auto", "trap", "pairwin", "window", "cta", "class"])
+@pytest.mark.parametrize("method", ["auto", "trap", "window", "class"])
 def test_photomosaic_pipeline_config2(method):
     I, T = pair("smooth", 512, 16)
     E_np = oracle_E("smooth", 512, 16)
@@ -338,25 +356,18 @@ def test_invalid_arguments_launch_nothing():
 def test_launch_count_increments():
     I, T = pair("smooth", 128, 8)
     n0 = pm.launch_count()
-    pm.photomosaic(dev(I), dev(T), 8, method="cta")
+    pm.photomosaic(dev(I), dev(T), 8, method="class")
     assert pm.launch_count() - n0 >= 5   # 2 pack + E + iota + search + cost
 
 
-@pytest.mark.parametrize("method", ["window", "pairwin"])
+@pytest.mark.parametrize("method", ["window"])
 @pytest.mark.parametrize("N,M", [(1600, 40), (1152, 32), (1440, 32), (224, 32), (280, 40)])
 def test_local_search_window_sizes(N, M, method):
     # S = 1600, 1296, 2025 (the second window tier, S in (1024, 2048]), 49, 49 -- grayscale noise
     _check_ls(oracle_E("noise", N, M, 1), method)
 
 
-@pytest.mark.parametrize("fam", ["smooth", "noise", "ties", "transposition", "identical", "shuffle"])
-@pytest.mark.parametrize("N,M", [(512, 16), (160, 8), (328, 8)])
-def test_local_search_pairwin_families(fam, N, M):
-    # S = 1024, 400, 1681 (odd)
-    _check_ls(oracle_E(fam, N, M), "pairwin")
-
-
-@pytest.mark.parametrize("method", ["window", "pairwin"])
+@pytest.mark.parametrize("method", ["window"])
 @pytest.mark.parametrize("S_side", [7, 31, 33, 45])
 def test_local_search_window_odd_mid(S_side, method):
     # odd S around the window tiers (49, 961, 1089, 2025)
@@ -458,20 +469,20 @@ def test_render_transposition_reproduces_target():
 @pytest.mark.parametrize("T", ["0", "1", "40", "1000000000"])
 @pytest.mark.parametrize("shape,fam", [((128, 8, 3), "smooth"), ((512, 16, 3), "smooth"), ((90, 10, 3), "smooth"),
                                        ((200, 5, 1), "noise"), ((128, 8, 3), "ties"), ((42, 6, 3), "transposition")])
-def test_sparse_rounds_parity(monkeypatch, cwalk, method, T, shape, fam):
-    monkeypatch.setenv("PM_LS_CWALK", cwalk)
-    monkeypatch.setenv("PM_LS_SPARSE_T", T)
+def test_sparse_rounds_parity(cwalk, method, T, shape, fam):
+    pm.tuning_set("ls_cwalk", int(cwalk))
+    pm.tuning_set("ls_sparse_T", int(T))
     _check_ls(oracle_E(fam, *shape), method)
 
 
 @pytest.mark.parametrize("cwalk", ["0", "1"])
 @pytest.mark.parametrize("gmem", ["0", "1"])
-def test_sparse_rounds_global_arrays_and_resume(monkeypatch, gmem, cwalk):
+def test_sparse_rounds_global_arrays_and_resume(gmem, cwalk):
     """Walk arrays in global memory (the S > 17K layout, forced), a resumed
     search and a max_rounds cut that lands inside the sparse stage."""
-    monkeypatch.setenv("PM_LS_SPARSE_GMEM", gmem)
-    monkeypatch.setenv("PM_LS_CWALK", cwalk)
-    monkeypatch.setenv("PM_LS_SPARSE_T", "1000000000")
+    pm.tuning_set("ls_sparse_gmem", int(gmem))
+    pm.tuning_set("ls_cwalk", int(cwalk))
+    pm.tuning_set("ls_sparse_T", 1000000000)
     E_np = oracle_E("smooth", 512, 16)
     _check_ls(E_np, "walk")
     for mr in (1, 2, 4):
@@ -485,8 +496,8 @@ def test_sparse_rounds_global_arrays_and_resume(monkeypatch, gmem, cwalk):
     _check_ls(E_np, "window", perm0=rng.permutation(E_np.shape[0]))
 
 
-def test_sparse_rounds_disabled_matches(monkeypatch):
-    monkeypatch.setenv("PM_LS_SPARSE", "0")
+def test_sparse_rounds_disabled_matches():
+    pm.tuning_set("ls_sparse", 0)
     _check_ls(oracle_E("smooth", 512, 16), "window")
     _check_ls(oracle_E("smooth", 128, 8), "class")
 
@@ -517,13 +528,13 @@ def test_walk_mailbox_overflow_falls_back_exactly():
     assert ref[3][0] >= 63
 
 
-def _check_trap(E_np):
+def _check_trap(E_np, cluster_forced=False):
     # the cluster mode is unsupported (PM_ERR_UNSUPPORTED) when the chunks do
     # not fit one cluster; every other outcome must match the oracle
     try:
         _check_ls(E_np, "trap")
     except pm.PMError as e:
-        if e.status != pm.PM_ERR_UNSUPPORTED or os.environ.get("PM_TRAP_CLUSTER") != "1":
+        if e.status != pm.PM_ERR_UNSUPPORTED or not cluster_forced:
             raise
         pytest.skip("chunks do not fit one cluster")
 
@@ -535,23 +546,23 @@ def _check_trap(E_np):
 @pytest.mark.parametrize("N,M,fam,W", [(128, 8, "smooth", 0), (512, 16, "smooth", 0), (512, 16, "ties", 7),
                                        (240, 8, "noise", 0), (336, 8, "smooth", 21), (128, 8, "transposition", 19)])
 @pytest.mark.parametrize("mode", ["0", "1"])
-def test_trap_every_round(variant, N, M, fam, W, mode, monkeypatch):
-    monkeypatch.setenv("PM_TRAP_V", str(variant))
-    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
-    monkeypatch.setenv("PM_LS_SPARSE", "0")
-    monkeypatch.setenv("PM_TRAP_W", str(W))
-    _check_trap(oracle_E(fam, N, M))
+def test_trap_every_round(variant, N, M, fam, W, mode):
+    pm.tuning_set("trap_variant", int(variant))
+    pm.tuning_set("trap_cluster", int(mode))
+    pm.tuning_set("ls_sparse", 0)
+    pm.tuning_set("trap_W", int(W))
+    _check_trap(oracle_E(fam, N, M), mode == "1")
 
 
 @pytest.mark.parametrize("cpc,variant", [(1, 0), (2, 0), (3, 1), (1, 3), (2, 4), (4, 2), (8, 1)])
 @pytest.mark.parametrize("mode", ["0", "1"])
-def test_trap_chunks_per_cta(cpc, variant, mode, monkeypatch):
-    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
-    monkeypatch.setenv("PM_TRAP_CPC", str(cpc))
-    monkeypatch.setenv("PM_TRAP_V", str(variant))
-    monkeypatch.setenv("PM_LS_SPARSE", "0")
+def test_trap_chunks_per_cta(cpc, variant, mode):
+    pm.tuning_set("trap_cluster", int(mode))
+    pm.tuning_set("trap_cpc", int(cpc))
+    pm.tuning_set("trap_variant", int(variant))
+    pm.tuning_set("ls_sparse", 0)
     # cluster mode holds every chunk in <= 16 CTAs: S = 1024 (16-64 chunks)
-    _check_trap(oracle_E("noise", 1024 if mode == "0" else 512, 16))
+    _check_trap(oracle_E("noise", 1024 if mode == "0" else 512, 16), mode == "1")
 
 
 @pytest.mark.parametrize("method", ["trap", "class", "window"])
@@ -569,13 +580,13 @@ def test_local_search_padded_leading_dimension(method):
 
 
 @pytest.mark.parametrize("variant,mode,vec", [("0", "0", "1"), ("0", "0", "0"), ("1", "1", "1"), ("3", "0", "1"), ("5", "0", "0")])
-def test_trap_every_round_config3(variant, mode, vec, monkeypatch):
+def test_trap_every_round_config3(variant, mode, vec):
     # S = 4096 with P = 768: pair-0 swaps at every u0 mod 4 (the 16-byte span offsets)
-    monkeypatch.setenv("PM_TRAP_V", variant)
-    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
-    monkeypatch.setenv("PM_TRAP_VEC", vec)
-    monkeypatch.setenv("PM_LS_SPARSE", "0")
-    _check_trap(oracle_E("smooth", 1024, 16))
+    pm.tuning_set("trap_variant", int(variant))
+    pm.tuning_set("trap_cluster", int(mode))
+    pm.tuning_set("trap_vec", int(vec))
+    pm.tuning_set("ls_sparse", 0)
+    _check_trap(oracle_E("smooth", 1024, 16), mode == "1")
 
 
 # ---- multi-GPU TRAP protocol (pm_local_search_multi_*): every rank of a world
@@ -594,8 +605,8 @@ def test_multi_rank_trap_emulated(N, M, fam, world):
 
 
 @pytest.mark.parametrize("variant", ["0", "5"])
-def test_multi_rank_trap_geometries(variant, monkeypatch):
-    monkeypatch.setenv("PM_TRAP_V", variant)
+def test_multi_rank_trap_geometries(variant):
+    pm.tuning_set("trap_variant", int(variant))
     E_np = oracle_E("smooth", 1024, 16)
     ref = oracle.local_search(E_np)
     out, rounds, swaps = pm.local_search_multi_emulated(dev(E_np), 3)
@@ -636,11 +647,60 @@ def test_multi_rank_trap_symmetric_memory_world1():
 
 
 @pytest.mark.parametrize("ep,mode", [("0", "1"), ("0", "0"), ("1", "0"), ("1", "1")])
-def test_trap_sigma_permuted_and_plain_row_staging(ep, mode, monkeypatch):
+def test_trap_sigma_permuted_and_plain_row_staging(ep, mode):
     # runs staged from the sigma-permuted copy of E (default while E is
     # L2-resident) or from E's rows directly: identical results
-    monkeypatch.setenv("PM_TRAP_EP", ep)
-    monkeypatch.setenv("PM_TRAP_CLUSTER", mode)
-    monkeypatch.setenv("PM_LS_SPARSE", "0")
-    _check_trap(oracle_E("smooth", 512, 16))
-    _check_trap(oracle_E("ties", 128, 8))
+    pm.tuning_set("trap_ep", int(ep))
+    pm.tuning_set("trap_cluster", int(mode))
+    pm.tuning_set("ls_sparse", 0)
+    _check_trap(oracle_E("smooth", 512, 16), mode == "1")
+    _check_trap(oracle_E("ties", 128, 8), mode == "1")
+
+
+# ------------------------------------------------------- failure paths -----
+def test_multi_rank_timeout_when_a_peer_never_runs():
+    # rank 0 of a world of 2 on this GPU; rank 1 is never launched.  Every
+    # cross-rank wait is bounded: rank 0 stops with PM_ERR_TIMEOUT instead of
+    # hanging, and the sparse rounds after it do not run
+    S = 1024
+    E = dev(oracle_E("smooth", 512, 16))
+    wsb = (pm.trap_workspace_bytes(S) + 255) // 256 * 256
+    bufs = [torch.zeros(wsb + 4 * S, dtype=torch.uint8, device=DEV) for _ in range(2)]
+    perms = [b[wsb:].view(torch.int32) for b in bufs]
+    for p_ in perms:
+        pm.init_identity(p_)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    with pm.tuning(trap_wait_ms=300):
+        pm.local_search_multi_async(E, [p_.data_ptr() for p_ in perms], [b.data_ptr() for b in bufs], 0, 2, res)
+        torch.cuda.synchronize()
+    assert int(res[0]) == pm.PM_ERR_TIMEOUT
+    # the device is still usable: a normal search right after is exact
+    _check_ls(oracle_E("smooth", 512, 16), "trap")
+
+
+def test_multi_rank_rejects_unsupported_before_enqueue():
+    E = torch.zeros((258, 258), dtype=torch.int32, device=DEV)
+    res = torch.full((3,), -5, dtype=torch.int64, device=DEV)
+    n0 = pm.launch_count()
+    with pytest.raises(pm.PMError) as ei:      # 129 pairs -> 5 chunks < world 8
+        pm.local_search_multi_async(E, [E.data_ptr()] * 8, [E.data_ptr()] * 8, 0, 8, res)
+    assert ei.value.status == pm.PM_ERR_UNSUPPORTED
+    assert int(res[0]) == -5 and pm.launch_count() == n0     # nothing enqueued
+
+
+def test_photomosaic_trap_odd_S_rejected_before_error_matrix():
+    I, T = pair("smooth", 90, 10)              # S = 81 (odd): TRAP does not take it
+    n0 = pm.launch_count()
+    with pytest.raises(pm.PMError) as ei:
+        pm.photomosaic(dev(I), dev(T), 10, method="trap")
+    assert ei.value.status == pm.PM_ERR_UNSUPPORTED and pm.launch_count() == n0
+
+
+def test_scratch_pool_trim():
+    E = dev(oracle_E("smooth", 512, 16))
+    pm.local_search(E)
+    torch.cuda.synchronize()
+    assert pm.scratch_reserved_bytes() > 0
+    pm.scratch_trim()
+    assert pm.scratch_reserved_bytes() == 0
+    _check_ls(oracle_E("smooth", 512, 16), "trap")           # the pool refills on demand

@@ -10,6 +10,9 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
 cfgs = [int(x) for x in (sys.argv[1:] or ["1", "2", "3"])]
 fams = os.environ.get("FAMS", "smooth").split(",")

@@ -1,9 +1,13 @@
+import sys
 """E-kernel (Step 2, Eq. 1) timing per BASELINE config: device-resident images,
 CUDA events, median of reps.  Development probe (the contract bench is bench.py)."""
 import os, statistics, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 from paper_conf_ipps_yangin17_b200 import pm, synth
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
 PEAK = 148 * 64 * 4 * 1.965e9          # VABSDIFF4.U8.ACC: 64 /clk/SM, 4 byte-absdiffs each
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["1", "2", "3", "4", "5"])]

@@ -7,9 +7,12 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["1", "2", "3"])]
-methods = sys.argv[2].split(",") if len(sys.argv) > 2 else ["window", "cta"]
+methods = sys.argv[2].split(",") if len(sys.argv) > 2 else ["trap", "window"]
 reps = max(1, int(os.environ.get("REPS", "5")))
 for cfg in cfgs:
     c = synth.CONFIGS[cfg]

@@ -9,6 +9,9 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["3", "4"])]
 worlds = [int(w) for w in (sys.argv[2].split(",") if len(sys.argv) > 2 else ["1", "2", "4", "8"])]

@@ -1,3 +1,4 @@
+import sys
 """NEXT-1 (SURVEY §8(f)): the paper's own workload grid -- grayscale (C = 1)
 N in {512, 1024, 2048} x S in {16^2, 32^2, 64^2} (Tables II-IV, P:346-422) --
 timed on this GPU with the same kernels: Step 2 (E) and Step 3 (Alg. 2, AUTO
@@ -8,6 +9,9 @@ import os, statistics, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 from paper_conf_ipps_yangin17_b200 import pm, synth
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
 # Table II (E, GPU s), Table III (approx. rearrangement, GPU s), Table IV (approx total, GPU s)
 PAPER = {(512, 16): (0.005, 0.012, 0.017), (512, 32): (0.017, 0.063, 0.081), (512, 64): (0.107, 0.343, 0.450),

@@ -1,3 +1,4 @@
+import sys
 """Small workload for compute-sanitizer: every kernel of libpm once (configs 1
 and a ragged odd shape), results checked against the oracle."""
 import os, sys
@@ -5,6 +6,9 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import oracle
 from paper_conf_ipps_yangin17_b200 import pm, synth
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 for (N, M, C) in [(128, 8, 3), (90, 10, 3)]:
     I, T = synth.make_pair("smooth", N, M, C, seed=1)
     dI, dT = torch.from_numpy(I).cuda(), torch.from_numpy(T).cuda()
@@ -12,10 +16,10 @@ for (N, M, C) in [(128, 8, 3), (90, 10, 3)]:
     Er = oracle.error_matrix(I, T, M)
     assert (E.cpu().numpy() == Er).all()
     ref = oracle.local_search(Er)
-    methods = os.environ.get("METHODS", "window,cta,class,pairwin").split(",")
+    methods = os.environ.get("METHODS", "trap,window,class,walk").split(",")
     perm = None
     for meth in methods:
-        if (meth == "pairwin" and E.shape[0] < 40) or (meth == "trap" and (E.shape[0] < 256 or E.shape[0] % 2)):
+        if (meth == "trap" and (E.shape[0] < 256 or E.shape[0] % 2)):
             continue
         perm, rounds, swaps, per, st = pm.local_search(E, method=meth)
         assert (perm.cpu().numpy() == ref[0]).all() and rounds == ref[1], meth

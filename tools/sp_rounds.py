@@ -1,9 +1,14 @@
+import sys
+import os
 """Per-round timing of the sparse rounds (needs tools/libpm_prof.so built
 with -DPM_LS_PROFILE).  Development probe: python tools/sp_rounds.py cfg method"""
 import ctypes, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 from paper_conf_ipps_yangin17_b200 import pm, synth
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 pm.LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), os.environ.get("PMLIB", "libpm_prof.so"))
 cfg = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 method = sys.argv[2] if len(sys.argv) > 2 else "window"

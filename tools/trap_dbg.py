@@ -8,6 +8,9 @@ import torch  # noqa: E402
 
 import oracle  # noqa: E402
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
 sizes = [(int(a), int(b)) for a, b in (x.split("/") for x in sys.argv[1].split(","))]
 for (N, M) in sizes:

@@ -10,8 +10,11 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+import _devknobs  # noqa: E402
+_devknobs.apply(pm)
 
-os.environ.setdefault("PM_TRAP_PROF", "1")
+pm.tuning_set("trap_prof", int(os.environ.get("PM_TRAP_PROF", "1")))
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["1", "2", "3"])]
 for cfg in cfgs:
     c = synth.CONFIGS[cfg]
