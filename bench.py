@@ -62,6 +62,7 @@ def parse():
     ap.add_argument("--family", default="smooth")
     ap.add_argument("--method", default="auto", choices=["auto", "trap", "class", "window", "walk"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-oracle", action="store_true", help="skip the oracle entirely (profiling runs)")
     ap.add_argument("--cpu-1t-rows", type=int, default=96,
                     help="rows of E in the one-thread oracle sample (extrapolated to S rows)")
     ap.add_argument("--ref-rows", type=int, default=1024,
@@ -525,12 +526,13 @@ def main():
         line, extra = bench_sharded(args, rank, world, local_rank)
     else:
         line, extra = bench_single(args, rank, world, local_rank)
-    if rank == 0:
+    if rank == 0 and not args.no_oracle:
         if world == 1:
             attach_oracle(line, extra, args)                 # cpu_baseline + parity
         elif not args.independent:
             args.no_cpu_baseline = True                      # cpu_baseline: rank 0 at N = 1 only
             attach_oracle(line, extra, args)                 # parity of the sharded result
+    if rank == 0:
         line["host"] = host_info()
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -70,7 +70,11 @@ struct TrapParams {
   int32_t vec;                 // 16-byte staging allowed (PM_TRAP_VEC, default 1)
   const int32_t* Ep;           // sigma-permuted copy of E (or NULL), leading dimension ldp
   int64_t ldp;
-  int32_t prof;                // PM_TRAP_PROF: CTA 0 thread 0 phase timers -> per_round[192..195]
+  int32_t prof;                // trap_prof: CTA 0 thread 0 phase timers -> per_round[192..196]
+  int32_t spec;                // speculative class steps (trap_spec, default 1)
+  int32_t prefetch;            // L2 prefetch of the next phases' E runs (trap_prefetch, default 1)
+  int32_t exp;
+  int32_t coal;                // warp-cooperative (coalesced) staging of the Ep runs
   unsigned int* bar;           // grid barrier counter (zeroed before launch)
   unsigned long long* rsw;     // [3] swaps per round, rotating (grid mode)
   LsResult* out;
@@ -92,9 +96,25 @@ struct TrapSmem {
   static constexpr int NC = 2 * T + 2;      // pair-0 light-cone tiles (at most)
   static constexpr int NU = (2 * T + 2 + 3 + 3) / 4 * 4;   // their span of E[g][u0 + z], z <= 2T+1
   static constexpr int UOFF = L * RS;       // cone rows follow the rows (one index space)
-  static constexpr int ints = (L * (4 + 1 + RS) + NC * NU + 3) / 4 * 4;   // int4 state + g + rows + cone rows
+  static constexpr int MOFF = UOFF + NC * NU;   // 3 rotating first-firing-class slots (speculative steps)
+  static constexpr int ints = (L * (4 + 1) + MOFF + 3 + 3) / 4 * 4;   // int4 state + g + rows + cone rows + slots
   static constexpr size_t bytes = sizeof(int32_t) * (size_t)ints;
 };
+
+constexpr int32_t kSpecB0 = 4;   // classes per speculative batch after a firing class (doubles while quiet)
+
+// Speculative class steps pay once firing classes are rare in a chunk's
+// trapezoid: a speculative iteration (batch test + first-class reduction +
+// apply, two barriers) costs ~3 chain steps (measured), so they
+// are used from the second round on, when the previous round's swaps put
+// fewer than ~1/8 firing pairs per class into an X-pair range (the previous
+// round's count over-estimates this round's).  mode: trap_spec (0 never,
+// 1 this rule, 2 always).  Results are identical either way.
+__device__ __forceinline__ bool spec_round(int32_t mode, int64_t prev_rs, int32_t X, int32_t ncls, int32_t npairs) {
+  if (mode == 2) return true;
+  if (mode != 1 || prev_rs < 0) return false;
+  return prev_rs * (int64_t)X * 8 < (int64_t)ncls * npairs;
+}
 
 __device__ __forceinline__ int32_t wrap_m(int32_t x, int32_t m) {
   x = x < 0 ? x + m : x;
@@ -129,6 +149,9 @@ __device__ __forceinline__ void stage_span(int32_t* dst, const int32_t* row, int
       cp_async4(dst + q, row + y);
     }
   }
+}
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
@@ -214,18 +237,34 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
                                           const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
                                           int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
                                           bool vec, unsigned long long* tprof,
-                                          const int32_t* __restrict__ Ep = nullptr, int64_t ldp = 0) {
+                                          const int32_t* __restrict__ Ep, int64_t ldp, bool spec, bool pf, int exp = 0,
+                                          bool coal = false) {
   using SM = TrapSmem<PPL, T>;
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
   const bool low = (C.a == 0);
   int32_t* s_U = s_E + SM::UOFF;
   // ---- one thread per local slot j (= local tile j): its state, then its
-  // tile's E row pieces, every copy independent of the others ----
-  for (int32_t j = gt; j < Lc; j += GT) {
-    const int32_t x = C.slot_of(j, u0, S);
-    int32_t g, d;
-    src(x, g, d);
+  // tile's E row pieces, every copy independent of the others.  Both slots'
+  // states are loaded before any copy is issued (two L2 round trips in
+  // flight together) ----
+  constexpr int NJ = (SM::L + GT - 1) / GT;   // slots per thread (2)
+  int32_t xs[NJ], gs[NJ], ds[NJ];
+  int32_t offA[NJ], offB[NJ];                 // coalesced staging: element offsets of the two runs in Ep
+#pragma unroll
+  for (int i = 0; i < NJ; ++i) {
+    const int32_t j = gt + i * GT;
+    xs[i] = 0; gs[i] = 0; ds[i] = 0;
+    if (j < Lc) {
+      xs[i] = C.slot_of(j, u0, S);
+      src(xs[i], gs[i], ds[i]);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < NJ; ++i) {
+    const int32_t j = gt + i * GT;
+    if (j >= Lc) continue;
+    const int32_t x = xs[i], g = gs[i], d = ds[i];
     s_g[j] = g;
     const bool fx = (x == S - 1);
     const int32_t ci = C.cone(j);
@@ -242,19 +281,64 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
                    : make_int4(j | (1 << 16), d, j * RS + (sp & 3), j * RS + SM::SP + (ss & 3) + 1);
       const int32_t* prow = Ep + (int64_t)g * ldp;
-      for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + q, prow + (sp & ~3) + q);
-      for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + SM::SP + q, prow + (ss & ~3) + q);
+      offA[i] = (int32_t)((int64_t)g * ldp + (sp & ~3));
+      offB[i] = (int32_t)((int64_t)g * ldp + (ss & ~3));
+      if (!(exp & 2) && !coal) {
+      if (!(exp & 16)) for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + q, prow + (sp & ~3) + q);
+      if (!(exp & 8)) for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + SM::SP + q, prow + (ss & ~3) + q);
+      }
+      if (pf && !fx) {
+        // the tile's partner runs of the next two phases continue this one
+        // (sigma(p0 + 2T) = sigma(p0) + T): pull them into L2 now, so the
+        // next stagings find them there if the tile stays (a hint only)
+        int32_t sn = sp + T;
+        sn = sn >= m ? sn - m : sn;
+        const int64_t nb = min((int64_t)(2 * SM::SPP * 4), 4 * (ldp - (sn & ~3))) & ~15ll;   // inside the row
+        if (nb >= 16) prefetch_l2(prow + (sn & ~3), (uint32_t)nb);
+      }
     } else {
       s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
                    : make_int4(j | (2 << 16), d, j * RS + (p0 & 3), j * RS + SM::SP + (s0 & 3) + 2);
       stage_span(dst, row, p0 & ~3, SM::SP, m, vec);
       stage_span(dst + SM::SP, row, s0 & ~3, SM::SP, m, vec);
+      if (pf && !fx) {   // columns p0 + 2T .. p0 + 4T + 4 of the plain row (stride-2 runs)
+        int32_t cn = p0 + 2 * T;
+        cn = cn >= m ? cn - m : cn;
+        const int32_t c16 = cn & ~3;
+        const int32_t nb = min(4 * (2 * T + 8), 4 * (m - c16)) & ~15;
+        if (vec && nb >= 16) prefetch_l2(row + c16, (uint32_t)nb);
+      }
     }
     cp_async4(dst + SM::CL, row + (S - 1));
     if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, vec);
   }
+  if (Ep && coal && !(exp & 2)) {
+    // warp-cooperative copies of the runs of the warp's 32 slots: lane l of
+    // copy `ins` moves 16-byte piece P = 32 ins + l of the warp's 64 runs, so
+    // one warp instruction covers ~3.5 whole runs (contiguous pieces, ~18
+    // sectors / ~8 lines) instead of 32 pieces of 32 different runs
+    constexpr int NP = SM::SPP / 4;           // 16-byte pieces per run
+    const int lane = gt & 31;
+    const int wbase = gt - lane;
+#pragma unroll
+    for (int i = 0; i < NJ; ++i) {
+#pragma unroll
+      for (int ins = 0; ins < 2 * NP; ++ins) {
+        const int P = ins * 32 + lane;
+        const int r = P / NP;                 // run of the warp: 2 per slot
+        const int q = P - r * NP;
+        const int sl = r >> 1;
+        const int32_t oA = __shfl_sync(0xffffffffu, offA[i], sl);
+        const int32_t oB = __shfl_sync(0xffffffffu, offB[i], sl);
+        const int32_t js = wbase + sl + i * GT;
+        if (js < Lc) cp_async16(s_E + js * RS + ((r & 1) ? SM::SP : 0) + 4 * q, Ep + ((r & 1) ? oB : oA) + 4 * q);
+      }
+    }
+  }
+  if (spec && gt < 3) s_E[SM::MOFF + gt] = INT32_MAX;
   cp_async_wait_all();
   group_sync(bar_id, GT);
+  if (exp & 4) return 0;
   unsigned long long t0 = tprof ? gtimer() : 0;
   // ---- Tp classes on the extended range: thread gt takes pair k = a + gt,
   // valid while t <= tmax (the trapezoid); its local slots are linear in t ----
@@ -269,27 +353,93 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
   }
   const int32_t tk = K - k, b1 = k - C.a, c1 = C.nA + m - C.a2 - k;   // j1 = t <= tk ? b1 + t : c1 - t
   const int32_t b2 = -k - C.a, c2 = C.nA + k - C.a2;                   // j2 = t >= k ? b2 + t : c2 - t
-  for (int32_t t = 0; t < Tp; ++t) {
-    if (t <= tmax) {
-      const int32_t j1 = (t <= tk) ? b1 + t : c1 - t;
-      const int32_t j2 = (k == 0) ? Lc - 1 : ((t >= k) ? b2 + t : c2 - t);
-      const int4 A = s_st[j1], B = s_st[j2];
-      const int32_t e_bu = s_E[B.z];
-      const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z];
-      const int32_t ia = A.x >> 16, ib = B.x >> 16;
-      const bool sw = A.y + B.y > e_bu + e_av;
-      int4 nA = sw ? make_int4(B.x, e_bu, B.w, B.z + ib) : make_int4(A.x, A.y, A.z + ia, A.w);
-      int4 nB = sw ? make_int4(A.x, e_av, A.w, A.z + ia) : make_int4(B.x, B.y, B.z + ib, B.w);
-      if (k == 0 && sw) {   // B leaves S-1 for slot u0+t (next partner u0+t+2), A enters S-1
-        const int32_t rb = SM::UOFF + C.cone(B.x & 0xffff) * SM::NU + (u0 & 3) + t + 2;
-        nA = make_int4((B.x & 0xffff) | (2 << 16), e_bu, rb, rb);
-        nB = make_int4((A.x & 0xffff) | (1 << 16), e_av, SM::UOFF + C.cone(A.x & 0xffff) * SM::NU + (u0 & 3) + t + 1, 0);
+  if (spec) {
+    // Speculative steps (exact).  The state of every slot is stored as of the
+    // last class that changed it, with its partner-entry index in the form
+    // z' = z - t * inc (z advances by inc per class while the slot does not
+    // swap), so class t >= tc can be tested on the state left by class tc-1
+    // directly: as long as no valid pair of classes [tc, t) fires, every slot
+    // a valid pair of class t reads is unchanged since tc (the trapezoid:
+    // valid pairs read only slots written by valid pairs).  Each iteration
+    // tests a batch of classes, takes the first class t* in which a valid
+    // pair fires, applies exactly the firing pairs of t* (the pairs of a class
+    // are disjoint) and resumes at t* + 1.  Quiet classes thus cost one
+    // parallel test instead of a dependent LDS -> LDS -> STS -> barrier step.
+    int32_t* s_first = s_E + SM::MOFF;   // reset before the staging barrier above
+    int32_t tc = 0, nb = kSpecB0;
+    uint32_t it = 0;
+    while (tc < Tp) {
+      const int32_t te = min(tc + nb, Tp);
+      const int32_t tl = min(te, tmax + 1);
+      int32_t myt = INT32_MAX, fj1 = 0, fj2 = 0, f_bu = 0, f_av = 0;
+      int4 fA = make_int4(0, 0, 0, 0), fB = fA;
+#pragma unroll 4
+      for (int32_t t = tc; t < tl; ++t) {
+        const int32_t j1 = (t <= tk) ? b1 + t : c1 - t;
+        const int32_t j2 = (k == 0) ? Lc - 1 : ((t >= k) ? b2 + t : c2 - t);
+        const int4 A = s_st[j1], B = s_st[j2];
+        const int32_t ia = A.x >> 16, ib = B.x >> 16;
+        const int32_t e_bu = s_E[B.z + t * ib];
+        const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z + t * ia];
+        if (myt == INT32_MAX && A.y + B.y > e_bu + e_av) {
+          myt = t; fj1 = j1; fj2 = j2; fA = A; fB = B; f_bu = e_bu; f_av = e_av;
+        }
       }
-      s_st[j1] = nA;
-      s_st[j2] = nB;
-      mysw += (sw && own) ? 1 : 0;
+      // first firing class of the chunk's valid trapezoid in [tc, te)
+      int32_t* slot = s_first + (it % 3u);
+      if (gt == 0) s_first[(it + 1) % 3u] = INT32_MAX;   // last read two iterations ago
+      const int32_t wmin = __reduce_min_sync(0xffffffffu, myt);
+      if ((gt & 31) == 0 && wmin != INT32_MAX) atomicMin(slot, wmin);
+      group_sync(bar_id, GT);
+      const int32_t ts = *slot;
+      ++it;
+      if (ts == INT32_MAX) {          // nothing fires in [tc, te): all decided
+        tc = te;
+        nb = min(2 * nb, (int32_t)T);
+        continue;
+      }
+      if (myt == ts) {                // apply class ts (state unchanged since tc)
+        const int32_t ia = fA.x >> 16, ib = fB.x >> 16;
+        int4 nA, nB;
+        if (k == 0) {                 // B leaves S-1 for slot u0+ts (next partner u0+ts+2), A enters S-1
+          const int32_t rb = SM::UOFF + C.cone(fB.x & 0xffff) * SM::NU + (u0 & 3) + ts + 2;
+          nA = make_int4((fB.x & 0xffff) | (2 << 16), f_bu, rb - 2 * (ts + 1), rb);
+          nB = make_int4((fA.x & 0xffff) | (1 << 16), f_av, SM::UOFF + C.cone(fA.x & 0xffff) * SM::NU + (u0 & 3), 0);
+        } else {
+          nA = make_int4(fB.x, f_bu, fB.w - (ts + 1) * ib, fB.z + (ts + 1) * ib);
+          nB = make_int4(fA.x, f_av, fA.w - (ts + 1) * ia, fA.z + (ts + 1) * ia);
+        }
+        s_st[fj1] = nA;
+        s_st[fj2] = nB;
+        mysw += own ? 1 : 0;
+      }
+      group_sync(bar_id, GT);
+      tc = ts + 1;
+      nb = kSpecB0;
     }
-    group_sync(bar_id, GT);
+  } else {
+    for (int32_t t = 0; t < Tp; ++t) {
+      if (t <= tmax) {
+        const int32_t j1 = (t <= tk) ? b1 + t : c1 - t;
+        const int32_t j2 = (k == 0) ? Lc - 1 : ((t >= k) ? b2 + t : c2 - t);
+        const int4 A = s_st[j1], B = s_st[j2];
+        const int32_t e_bu = s_E[B.z];
+        const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z];
+        const int32_t ia = A.x >> 16, ib = B.x >> 16;
+        const bool sw = A.y + B.y > e_bu + e_av;
+        int4 nA = sw ? make_int4(B.x, e_bu, B.w, B.z + ib) : make_int4(A.x, A.y, A.z + ia, A.w);
+        int4 nB = sw ? make_int4(A.x, e_av, A.w, A.z + ia) : make_int4(B.x, B.y, B.z + ib, B.w);
+        if (k == 0 && sw) {   // B leaves S-1 for slot u0+t (next partner u0+t+2), A enters S-1
+          const int32_t rb = SM::UOFF + C.cone(B.x & 0xffff) * SM::NU + (u0 & 3) + t + 2;
+          nA = make_int4((B.x & 0xffff) | (2 << 16), e_bu, rb, rb);
+          nB = make_int4((A.x & 0xffff) | (1 << 16), e_av, SM::UOFF + C.cone(A.x & 0xffff) * SM::NU + (u0 & 3) + t + 1, 0);
+        }
+        s_st[j1] = nA;
+        s_st[j2] = nB;
+        mysw += (sw && own) ? 1 : 0;
+      }
+      group_sync(bar_id, GT);
+    }
   }
   if (tprof) *tprof += gtimer() - t0;
   return mysw;
@@ -365,10 +515,13 @@ k_ls_trap(const TrapParams p) {
   const unsigned pblk = p.prof == 2 ? nblk - 1 : (p.prof == 3 ? nblk / 2 : 0);
   const bool prof = p.prof && blockIdx.x == pblk && threadIdx.x == 0 && p.max_log >= 200;
   unsigned long long t_ld = 0, t_st = 0, t_bar = 0, t_pub = 0, n_ph = 0, tq = prof ? gtimer() : 0;
+  const unsigned long long t_start0 = tq;
   const int npass = (p.nchunks + ngrp_tot - 1) / ngrp_tot;
   uint32_t nph_cl = 0;   // cluster mode: phases completed (mbarrier parity)
   uint32_t qph = 0;      // grid mode: phases completed
+  int64_t prev_rs = -1;   // swaps of the previous round (-1: none yet)
   for (;;) {
+    const bool spec = spec_round(p.spec, prev_rs, X, ncls, K + 1);
     if (!CLU && blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
@@ -389,12 +542,12 @@ k_ls_trap(const TrapParams p) {
             const int2* rr = rep + cur * S;
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { const int2 v = rr[x]; g = v.x; d = v.y; },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
           } else {
             const int bi = p.nbsync ? (int)(qph % 3u) : cur;
             const int32_t* __restrict__ rc = bi == 0 ? p.rbuf[0] : (bi == 1 ? p.rbuf[1] : p.rbuf[2]);
             const int32_t* __restrict__ dc = bi == 0 ? p.dbuf[0] : (bi == 1 ? p.dbuf[1] : p.dbuf[2]);
-            if (p.nbsync && qph > 0) {
+            if (p.nbsync && qph > 0 && !(p.exp & 1)) {
               // the neighbour chunks' slots of phase qph - 1 (W >= 2T: every
               // reader of this buffer's previous generation is within two
               // chunks, and those finished it before our neighbours did theirs)
@@ -413,7 +566,7 @@ k_ls_trap(const TrapParams p) {
             }
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
           // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
@@ -498,7 +651,9 @@ k_ls_trap(const TrapParams p) {
     }
     __syncthreads();
     const int64_t rs = (int64_t)s_rs;
+    prev_rs = rs;
     if (blockIdx.x == 0 && threadIdx.x == 0 && rounds < p.max_log) p.per_round[rounds] = rs;
+    if (prof && rounds < 32) p.per_round[224 + rounds] = (int64_t)gtimer();   // round end times (trap_prof)
     rounds += 1;
     total += rs;
     __syncthreads();   // (a CTA's s_rsw slot is rewritten three rounds later)
@@ -510,6 +665,7 @@ k_ls_trap(const TrapParams p) {
     }
   }
   if (prof) {
+    p.per_round[197] = (int64_t)t_start0;
     p.per_round[192] = (int64_t)(t_ld - t_st); p.per_round[193] = (int64_t)t_st;
     p.per_round[194] = (int64_t)t_bar; p.per_round[195] = (int64_t)n_ph;
     p.per_round[196] = (int64_t)t_pub;
@@ -655,6 +811,10 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.bar = bar; hp.rsw = rsw;
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.prof = knob("trap_prof", 0);
+  hp.exp = knob("trap_exp", 0);
+  hp.coal = knob("trap_coal", 1);
+  hp.spec = knob("trap_spec", 0);
+  hp.prefetch = knob("trap_prefetch", 0);
   // sigma-permuted rows (the runs become contiguous: 5 instead of 9 16-byte
   // pieces per run at T = 16 from L2, dense sectors instead of stride-2 ones
   // from HBM)
@@ -667,6 +827,7 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
     PM_CUDA_TRY(pm::scratch_alloc(&ep.p, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
     PM_CUDA_TRY(launch_permute_cols(E, ldE, ep.as<int32_t>(), ldp, S, m, ext, st));
     hp.Ep = ep.as<int32_t>(); hp.ldp = ldp;
+    if ((int64_t)S * ldp >= (1ll << 31)) hp.coal = 0;   // int32 element offsets
   }
   // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
@@ -724,6 +885,9 @@ struct TrapMultiParams {
   int64_t* per_round;
   int32_t* handoff;               // the first rank's sparse-round flag (or NULL)
   int32_t sparse_T;
+  int32_t spec;                   // speculative class steps
+  int32_t prefetch;               // L2 prefetch of the next phases' E runs
+  int32_t coal;                   // coalesced staging of the Ep runs
   unsigned long long wait_ns;     // bound of every cross-rank wait
 };
 
@@ -838,7 +1002,9 @@ k_ls_trap_mr(const TrapMultiParams p) {
   int64_t total = 0;
   int status = PM_OK;
   unsigned int xtarget = 0;
+  int64_t prev_rs = -1;
   while (ok) {
+    const bool spec = spec_round(p.spec, prev_rs, X, ncls, K + 1);
     if (leader) me.rtot[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls && ok; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
@@ -868,7 +1034,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
           const int32_t* __restrict__ dc = me.dbuf[bi];
           mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
                                      [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
-                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp);
+                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp, spec, p.prefetch, 0, p.coal);
           // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
           int32_t own[3];
           int nown = 0;
@@ -939,6 +1105,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
     if (threadIdx.x == 0) s_rs = ld_acquire_sys64(me.rtot + rounds % 3);
     __syncthreads();
     const int64_t rs = (int64_t)s_rs;
+    prev_rs = rs;
     if (leader && r == p.rank0 && rounds < p.max_log) p.per_round[rounds] = rs;
     rounds += 1;
     total += rs;
@@ -1032,7 +1199,11 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.handoff = handoff; hp.sparse_T = sparse_T;
   hp.ldp = ldp;
+  const bool coal_ok = (int64_t)S * ldp < (1ll << 31);
   hp.wait_ns = (unsigned long long)knob("trap_wait_ms", 20000) * 1000000ull;
+  hp.spec = knob("trap_spec", 0);
+  hp.prefetch = knob("trap_prefetch", 0);
+  hp.coal = coal_ok ? knob("trap_coal", 1) : 0;
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
   int max_cpc = (int)((size_t)optin / SM::bytes);

@@ -554,6 +554,23 @@ def test_trap_every_round(variant, N, M, fam, W, mode):
     _check_trap(oracle_E(fam, N, M), mode == "1")
 
 
+@pytest.mark.parametrize("spec", [0, 1, 2])
+@pytest.mark.parametrize("variant", [0, 1, 3, 5])
+@pytest.mark.parametrize("N,M,fam", [(512, 16, "smooth"), (512, 16, "ties"), (336, 8, "smooth"), (1024, 16, "smooth")])
+@pytest.mark.parametrize("mode", ["0", "1"])
+def test_trap_speculative_steps(spec, variant, N, M, fam, mode):
+    # speculative class steps (batches of classes tested on the state of the
+    # batch start, first firing class applied exactly): off, after quiet
+    # rounds (default), every round -- with and without sparse rounds after
+    pm.tuning_set("trap_spec", spec)
+    pm.tuning_set("trap_variant", variant)
+    pm.tuning_set("trap_cluster", int(mode))
+    E_np = oracle_E(fam, N, M)
+    _check_trap(E_np, mode == "1")
+    pm.tuning_set("ls_sparse", 0)
+    _check_trap(E_np, mode == "1")
+
+
 @pytest.mark.parametrize("cpc,variant", [(1, 0), (2, 0), (3, 1), (1, 3), (2, 4), (4, 2), (8, 1)])
 @pytest.mark.parametrize("mode", ["0", "1"])
 def test_trap_chunks_per_cta(cpc, variant, mode):

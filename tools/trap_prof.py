@@ -1,6 +1,7 @@
-"""TRAP phase profile (PM_TRAP_PROF=1): block 0 / warp 0 time split per phase
-into staging (state + E runs), class steps, write-back + grid barrier.
-Development probe.  Usage: PM_TRAP_PROF=1 python tools/trap_prof.py [cfgs]"""
+"""TRAP phase profile (trap_prof=1): block 0 / warp 0 time split per phase
+into staging (state + E runs), class steps, write-back + grid barrier, and
+the duration of every TRAP round.  Development probe.
+Usage: PM_TRAP_PROF=1 [PM_TRAP_SPEC=0|1|2] python tools/trap_prof.py [cfgs]"""
 import ctypes
 import os
 import sys
@@ -27,7 +28,11 @@ for cfg in cfgs:
         r, sw = ctypes.c_int32(0), ctypes.c_int64(0)
         st = pm.lib().pm_local_search_ex(E.data_ptr(), E.stride(0), S, perm.data_ptr(), 0, pm.METHODS["trap"],
                                          ctypes.byref(r), ctypes.byref(sw), per.ctypes.data, 256, None)
-    ld, stp, bar, nph, pub = per[192:197]
+    ld, stp, bar, nph, pub, t0 = per[192:198]
     nph = max(int(nph), 1)
+    ends = [int(x) for x in per[224:256] if x > 0]
+    rt = np.diff([int(t0)] + ends) / 1e3
     print(f"cfg{cfg} S={S} st={st} rounds={r.value} phases={nph} per phase: stage {ld/nph:.0f} ns, "
-          f"steps {stp/nph:.0f} ns, publish {pub/nph:.0f} ns, publish+barrier {bar/nph:.0f} ns; total {(ld+stp+bar)/1e6:.3f} ms", flush=True)
+          f"steps {stp/nph:.0f} ns, publish {pub/nph:.0f} ns, publish+barrier {bar/nph:.0f} ns; total "
+          f"{(ld+stp+bar)/1e6:.3f} ms; TRAP rounds (us) {np.round(rt, 1).tolist()} swaps {per[:len(rt)].tolist()}",
+          flush=True)
