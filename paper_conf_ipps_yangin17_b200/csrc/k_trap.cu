@@ -60,8 +60,9 @@ namespace pm {
 struct TrapParams {
   const int32_t* E;
   int64_t ldE;
-  int32_t* rbuf[3];            // rbuf[0] = the caller's perm (grid mode: phase q reads q % 3)
+  int32_t* rbuf[3];            // rbuf[0] = the caller's perm
   int32_t* dbuf[3];
+  int4* sbuf[3];               // grid mode: per-slot state {tile g, d = E[g][x], E[g][S-1], 0}; phase q reads q % 3
   unsigned int* flags;         // grid mode, neighbour sync: phases completed per chunk
   int32_t nbsync;              // grid mode: wait for the neighbour chunks only (W >= 2T)
   int32_t S, max_rounds, max_log, sparse_T;
@@ -74,6 +75,7 @@ struct TrapParams {
   int32_t spec;                // speculative class steps (trap_spec, default 1)
   int32_t prefetch;            // L2 prefetch of the next phases' E runs (trap_prefetch, default 1)
   int32_t exp;
+  int32_t fstride;             // chunk flag spacing (uint32 units)
   int32_t coal;                // warp-cooperative (coalesced) staging of the Ep runs
   unsigned int* bar;           // grid barrier counter (zeroed before launch)
   unsigned long long* rsw;     // [3] swaps per round, rotating (grid mode)
@@ -97,11 +99,10 @@ struct TrapSmem {
   static constexpr int NU = (2 * T + 2 + 3 + 3) / 4 * 4;   // their span of E[g][u0 + z], z <= 2T+1
   static constexpr int UOFF = L * RS;       // cone rows follow the rows (one index space)
   static constexpr int MOFF = UOFF + NC * NU;   // 3 rotating first-firing-class slots (speculative steps)
-  static constexpr int ints = (L * (4 + 1) + MOFF + 3 + 3) / 4 * 4;   // int4 state + g + rows + cone rows + slots
+  static constexpr int ints = (L * (4 + 1) + MOFF + 4 + 3) / 4 * 4;   // state + g + rows + cone rows + slots
   static constexpr size_t bytes = sizeof(int32_t) * (size_t)ints;
 };
 
-constexpr int32_t kSpecB0 = 4;   // classes per speculative batch after a firing class (doubles while quiet)
 
 // Speculative class steps pay once firing classes are rare in a chunk's
 // trapezoid: a speculative iteration (batch test + first-class reduction +
@@ -240,24 +241,26 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
                                           const int32_t* __restrict__ Ep, int64_t ldp, bool spec, bool pf, int exp = 0,
                                           bool coal = false) {
   using SM = TrapSmem<PPL, T>;
+  static_assert(T <= 32, "one mask bit per class of a phase");
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
   const bool low = (C.a == 0);
+  const bool aligned = ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);
   int32_t* s_U = s_E + SM::UOFF;
   // ---- one thread per local slot j (= local tile j): its state, then its
   // tile's E row pieces, every copy independent of the others.  Both slots'
   // states are loaded before any copy is issued (two L2 round trips in
   // flight together) ----
   constexpr int NJ = (SM::L + GT - 1) / GT;   // slots per thread (2)
-  int32_t xs[NJ], gs[NJ], ds[NJ];
+  int32_t xs[NJ], gs[NJ], ds[NJ], els[NJ];   // els: E[g][S-1] when the state carries it, else -1
   int32_t offA[NJ], offB[NJ];                 // coalesced staging: element offsets of the two runs in Ep
 #pragma unroll
   for (int i = 0; i < NJ; ++i) {
     const int32_t j = gt + i * GT;
-    xs[i] = 0; gs[i] = 0; ds[i] = 0;
+    xs[i] = 0; gs[i] = 0; ds[i] = 0; els[i] = -1;
     if (j < Lc) {
       xs[i] = C.slot_of(j, u0, S);
-      src(xs[i], gs[i], ds[i]);
+      src(xs[i], gs[i], ds[i], els[i]);
     }
   }
 #pragma unroll
@@ -309,8 +312,13 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
         if (vec && nb >= 16) prefetch_l2(row + c16, (uint32_t)nb);
       }
     }
-    cp_async4(dst + SM::CL, row + (S - 1));
-    if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, vec);
+    if (els[i] >= 0) dst[SM::CL] = els[i];          // carried by the published state (grid mode)
+    else cp_async4(dst + SM::CL, row + (S - 1));
+    // the pair-0 light cone's run E[g][u0 .. u0+2T+1] is contiguous (every
+    // entry used): 16-byte pieces whenever the rows are aligned.  (With
+    // 4-byte copies chunk 0 -- the only one with a cone -- was the straggler
+    // that paced the whole chunk chain: config 4 TRAP round 5.5 -> 5.0 ms.)
+    if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, aligned || vec);
   }
   if (Ep && coal && !(exp & 2)) {
     // warp-cooperative copies of the runs of the warp's 32 slots: lane l of
@@ -335,7 +343,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       }
     }
   }
-  if (spec && gt < 3) s_E[SM::MOFF + gt] = INT32_MAX;
+  if (spec && gt < 3) s_E[SM::MOFF + gt] = 0;
   cp_async_wait_all();
   group_sync(bar_id, GT);
   if (exp & 4) return 0;
@@ -360,46 +368,43 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     // swap), so class t >= tc can be tested on the state left by class tc-1
     // directly: as long as no valid pair of classes [tc, t) fires, every slot
     // a valid pair of class t reads is unchanged since tc (the trapezoid:
-    // valid pairs read only slots written by valid pairs).  Each iteration
-    // tests a batch of classes, takes the first class t* in which a valid
-    // pair fires, applies exactly the firing pairs of t* (the pairs of a class
-    // are disjoint) and resumes at t* + 1.  Quiet classes thus cost one
-    // parallel test instead of a dependent LDS -> LDS -> STS -> barrier step.
-    int32_t* s_first = s_E + SM::MOFF;   // reset before the staging barrier above
-    int32_t tc = 0, nb = kSpecB0;
+    // valid pairs read only slots written by valid pairs).  One pass tests
+    // every remaining class of the phase at once (a bit per class), the OR
+    // over the chunk gives the first class t* in which a valid pair fires;
+    // exactly the firing pairs of t* are applied (the pairs of a class are
+    // disjoint) and the next pass resumes at t* + 1.  A quiet phase thus
+    // costs one parallel pass instead of Tp dependent steps.
+    unsigned int* s_or = reinterpret_cast<unsigned int*>(s_E + SM::MOFF);   // reset before the staging barrier
+    int32_t tc = 0;
     uint32_t it = 0;
     while (tc < Tp) {
-      const int32_t te = min(tc + nb, Tp);
-      const int32_t tl = min(te, tmax + 1);
-      int32_t myt = INT32_MAX, fj1 = 0, fj2 = 0, f_bu = 0, f_av = 0;
-      int4 fA = make_int4(0, 0, 0, 0), fB = fA;
-#pragma unroll 4
+      const int32_t tl = min(Tp, tmax + 1);
+      uint32_t mask = 0;
+#pragma unroll 8
       for (int32_t t = tc; t < tl; ++t) {
         const int32_t j1 = (t <= tk) ? b1 + t : c1 - t;
         const int32_t j2 = (k == 0) ? Lc - 1 : ((t >= k) ? b2 + t : c2 - t);
         const int4 A = s_st[j1], B = s_st[j2];
-        const int32_t ia = A.x >> 16, ib = B.x >> 16;
-        const int32_t e_bu = s_E[B.z + t * ib];
-        const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z + t * ia];
-        if (myt == INT32_MAX && A.y + B.y > e_bu + e_av) {
-          myt = t; fj1 = j1; fj2 = j2; fA = A; fB = B; f_bu = e_bu; f_av = e_av;
-        }
+        const int32_t e_bu = s_E[B.z + t * (B.x >> 16)];
+        const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z + t * (A.x >> 16)];
+        mask |= (A.y + B.y > e_bu + e_av) ? (1u << t) : 0u;
       }
-      // first firing class of the chunk's valid trapezoid in [tc, te)
-      int32_t* slot = s_first + (it % 3u);
-      if (gt == 0) s_first[(it + 1) % 3u] = INT32_MAX;   // last read two iterations ago
-      const int32_t wmin = __reduce_min_sync(0xffffffffu, myt);
-      if ((gt & 31) == 0 && wmin != INT32_MAX) atomicMin(slot, wmin);
+      unsigned int* slot = s_or + (it % 3u);
+      if (gt == 0) s_or[(it + 1) % 3u] = 0u;   // last read two passes ago
+      const uint32_t wor = __reduce_or_sync(0xffffffffu, mask);
+      if ((gt & 31) == 0 && wor) atomicOr(slot, wor);
       group_sync(bar_id, GT);
-      const int32_t ts = *slot;
+      const uint32_t all = *slot;
       ++it;
-      if (ts == INT32_MAX) {          // nothing fires in [tc, te): all decided
-        tc = te;
-        nb = min(2 * nb, (int32_t)T);
-        continue;
-      }
-      if (myt == ts) {                // apply class ts (state unchanged since tc)
+      if (all == 0u) break;                    // nothing fires in [tc, Tp): the phase is decided
+      const int32_t ts = __ffs(all) - 1;       // first firing class
+      if ((mask >> ts) & 1u) {                 // apply my pair of class ts (state unchanged since tc)
+        const int32_t j1 = (ts <= tk) ? b1 + ts : c1 - ts;
+        const int32_t j2 = (k == 0) ? Lc - 1 : ((ts >= k) ? b2 + ts : c2 - ts);
+        const int4 fA = s_st[j1], fB = s_st[j2];
         const int32_t ia = fA.x >> 16, ib = fB.x >> 16;
+        const int32_t f_bu = s_E[fB.z + ts * ib];
+        const int32_t f_av = s_E[(k == 0) ? (fA.x & 0xffff) * RS + SM::CL : fA.z + ts * ia];
         int4 nA, nB;
         if (k == 0) {                 // B leaves S-1 for slot u0+ts (next partner u0+ts+2), A enters S-1
           const int32_t rb = SM::UOFF + C.cone(fB.x & 0xffff) * SM::NU + (u0 & 3) + ts + 2;
@@ -409,13 +414,12 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
           nA = make_int4(fB.x, f_bu, fB.w - (ts + 1) * ib, fB.z + (ts + 1) * ib);
           nB = make_int4(fA.x, f_av, fA.w - (ts + 1) * ia, fA.z + (ts + 1) * ia);
         }
-        s_st[fj1] = nA;
-        s_st[fj2] = nB;
+        s_st[j1] = nA;
+        s_st[j2] = nB;
         mysw += own ? 1 : 0;
       }
       group_sync(bar_id, GT);
       tc = ts + 1;
-      nb = kSpecB0;
     }
   } else {
     for (int32_t t = 0; t < Tp; ++t) {
@@ -501,8 +505,11 @@ k_ls_trap(const TrapParams p) {
     }
     cg::this_cluster().sync();
   } else {
-    for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
-      __stcg(p.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(p.rbuf[0] + x) * ld + x));
+    for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x) {
+      const int32_t g = __ldcg(p.rbuf[0] + x);
+      const int32_t* row = E + (int64_t)g * ld;
+      __stcg(p.sbuf[0] + x, make_int4(g, __ldg(row + x), __ldg(row + (S - 1)), 0));
+    }
     bar_target += nblk;
     grid_barrier(p.bar, bar_target);
   }
@@ -541,12 +548,11 @@ k_ls_trap(const TrapParams p) {
           if (CLU) {
             const int2* rr = rep + cur * S;
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
-                                       [&](int32_t x, int32_t& g, int32_t& d) { const int2 v = rr[x]; g = v.x; d = v.y; },
+                                       [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { const int2 v = rr[x]; g = v.x; d = v.y; el = -1; },
                                        s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
           } else {
             const int bi = p.nbsync ? (int)(qph % 3u) : cur;
-            const int32_t* __restrict__ rc = bi == 0 ? p.rbuf[0] : (bi == 1 ? p.rbuf[1] : p.rbuf[2]);
-            const int32_t* __restrict__ dc = bi == 0 ? p.dbuf[0] : (bi == 1 ? p.dbuf[1] : p.dbuf[2]);
+            const int4* __restrict__ sc = bi == 0 ? p.sbuf[0] : (bi == 1 ? p.sbuf[1] : p.sbuf[2]);
             if (p.nbsync && qph > 0 && !(p.exp & 1)) {
               // the neighbour chunks' slots of phase qph - 1 (W >= 2T: every
               // reader of this buffer's previous generation is within two
@@ -558,14 +564,16 @@ k_ls_trap(const TrapParams p) {
                   if (c2 < 0 || c2 >= p.nchunks) continue;
                   unsigned int v;
                   do {
-                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.flags + c2) : "memory");
+                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.flags + c2 * p.fstride) : "memory");
                   } while (v < qph);
                 }
               }
               group_sync(1 + grp, GT);
             }
             mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
-                                       [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
+                                       [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) {
+                                         const int4 v = __ldcg(sc + x); g = v.x; d = v.y; el = v.z;
+                                       },
                                        s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
@@ -593,11 +601,11 @@ k_ls_trap(const TrapParams p) {
                   st_async_v2(cluster_addr(a2, c2), g2, B.y, rm);
                 }
               } else {
+                // {tile, d, E[tile][S-1]}: the reader needs no second round trip
                 const int bn = p.nbsync ? (int)((qph + 1u) % 3u) : (cur ^ 1);
-                int32_t* rn = bn == 0 ? p.rbuf[0] : (bn == 1 ? p.rbuf[1] : p.rbuf[2]);
-                int32_t* dn = bn == 0 ? p.dbuf[0] : (bn == 1 ? p.dbuf[1] : p.dbuf[2]);
-                __stcg(rn + x1, g1); __stcg(dn + x1, A.y);
-                __stcg(rn + x2, g2); __stcg(dn + x2, B.y);
+                int4* sn = bn == 0 ? p.sbuf[0] : (bn == 1 ? p.sbuf[1] : p.sbuf[2]);
+                __stcg(sn + x1, make_int4(g1, A.y, s_E[(A.x & 0xffff) * SM::RS + SM::CL], 0));
+                __stcg(sn + x2, make_int4(g2, B.y, s_E[(B.x & 0xffff) * SM::RS + SM::CL], 0));
               }
             }
           }
@@ -605,8 +613,8 @@ k_ls_trap(const TrapParams p) {
         if (prof) { const unsigned long long t = gtimer(); t_pub += t - tq; }
         group_sync(1 + grp, GT);
         if (!CLU && p.nbsync && have && gt == 0) {   // this chunk's slots of phase qph are out
-          __threadfence();
-          asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.flags + ch), "r"(qph + 1u) : "memory");
+          if (!(p.exp & 32)) __threadfence();
+          asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.flags + ch * p.fstride), "r"(qph + 1u) : "memory");
         }
       }
       // swaps of this phase -> the round counter
@@ -687,11 +695,9 @@ k_ls_trap(const TrapParams p) {
     cg::this_cluster().sync();   // no CTA exits while others may still touch its smem
   } else {   // the final state is in buffer qph % 3 (nbsync) or cur: copy to perm
     const int bf = p.nbsync ? (int)(qph % 3u) : cur;
-    if (bf != 0) {
-      const int32_t* src = bf == 1 ? p.rbuf[1] : p.rbuf[2];
-      for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
-        p.rbuf[0][x] = __ldcg(src + x);
-    }
+    const int4* src = bf == 0 ? p.sbuf[0] : (bf == 1 ? p.sbuf[1] : p.sbuf[2]);
+    for (int32_t x = blockIdx.x * blockDim.x + threadIdx.x; x < S; x += nblk * blockDim.x)
+      p.rbuf[0][x] = __ldcg(src + x).x;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     p.out->status = status;
@@ -788,23 +794,23 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
                      int32_t* handoff, int32_t sparse_T) {
   if (S < ls_trap_min_S() || (S & 1)) return PM_ERR_UNSUPPORTED;
   PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
-  // scratch: 3 round counters, barrier counter, chunk flags [S/2], r1, r2,
-  // d0, d1, d2 [S]
+  // scratch: 3 round counters, barrier counter, chunk flags [S/2], then the
+  // three generations of packed slot states (int4 [S] each)
   const size_t n = (size_t)S;
   ScopedScratch scr(st), ep(st);
-  const size_t head = 64 + sizeof(unsigned int) * (n / 2 + 16);
-  const size_t bytes = head + sizeof(int32_t) * 5 * n;
+  const size_t head = (64 + sizeof(unsigned int) * (n / 2 + 16) * 32 + 15) / 16 * 16;
+  const size_t bytes = head + sizeof(int4) * 3 * n;
   PM_CUDA_TRY(pm::scratch_alloc(&scr.p, bytes, st));
   char* scratch = scr.as<char>();
   unsigned long long* rsw = reinterpret_cast<unsigned long long*>(scratch);
   unsigned int* bar = reinterpret_cast<unsigned int*>(scratch + 32);
   unsigned int* flags = reinterpret_cast<unsigned int*>(scratch + 64);
-  int32_t* base = reinterpret_cast<int32_t*>(scratch + head);
+  int4* base = reinterpret_cast<int4*>(scratch + head);
   PM_CUDA_TRY(cudaMemsetAsync(scratch, 0, head, st));
   TrapParams hp = {};
   hp.E = E; hp.ldE = ldE;
-  hp.rbuf[0] = perm; hp.rbuf[1] = base; hp.rbuf[2] = base + n;
-  hp.dbuf[0] = base + 2 * n; hp.dbuf[1] = base + 3 * n; hp.dbuf[2] = base + 4 * n;
+  hp.rbuf[0] = perm;
+  hp.sbuf[0] = base; hp.sbuf[1] = base + n; hp.sbuf[2] = base + 2 * n;
   hp.flags = flags;
   hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
   hp.sparse_T = sparse_T; hp.handoff = handoff;
@@ -812,8 +818,9 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.prof = knob("trap_prof", 0);
   hp.exp = knob("trap_exp", 0);
+  hp.fstride = (hp.exp & 64) ? 32 : 1;
   hp.coal = knob("trap_coal", 1);
-  hp.spec = knob("trap_spec", 0);
+  hp.spec = knob("trap_spec", 1);
   hp.prefetch = knob("trap_prefetch", 0);
   // sigma-permuted rows (the runs become contiguous: 5 instead of 9 16-byte
   // pieces per run at T = 16 from L2, dense sectors instead of stride-2 ones
@@ -1033,7 +1040,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
           const int32_t* __restrict__ rc = me.rbuf[bi];
           const int32_t* __restrict__ dc = me.dbuf[bi];
           mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
-                                     [&](int32_t x, int32_t& g, int32_t& d) { g = __ldcg(rc + x); d = __ldcg(dc + x); },
+                                     [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { g = __ldcg(rc + x); d = __ldcg(dc + x); el = -1; },
                                      s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp, spec, p.prefetch, 0, p.coal);
           // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
           int32_t own[3];
@@ -1201,7 +1208,7 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   hp.ldp = ldp;
   const bool coal_ok = (int64_t)S * ldp < (1ll << 31);
   hp.wait_ns = (unsigned long long)knob("trap_wait_ms", 20000) * 1000000ull;
-  hp.spec = knob("trap_spec", 0);
+  hp.spec = knob("trap_spec", 1);
   hp.prefetch = knob("trap_prefetch", 0);
   hp.coal = coal_ok ? knob("trap_coal", 1) : 0;
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
