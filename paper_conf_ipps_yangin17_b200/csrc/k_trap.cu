@@ -84,37 +84,43 @@ struct TrapParams {
   int32_t* handoff;
 };
 
-template <int PPL, int T>
+template <int PPL, int T, bool EP>
 struct TrapSmem {
   static constexpr int X = 32 * PPL;        // pairs of an extended range
   static constexpr int L = 2 * X;           // slots (= tiles) of an extended range
-  // staged row of local tile i: span0 [0, SP) holds E[g][(p0 & ~3) + q] and
-  // span1 [SP, 2SP) E[g][(s0 & ~3) + q] (16-byte copies; the runs p0 + 2j,
-  // s0 + 2j, j <= T, are their entries (p0 & 3) + 2j), E[g][S-1] at CL
-  static constexpr int SP = (2 * T + 4 + 3) / 4 * 4;
-  static constexpr int SPP = (T + 1 + 3 + 3) / 4 * 4;   // the same runs from sigma-permuted rows
+  // staged row of local tile i: span0 [0, SP) holds the tile's partner run,
+  // span1 [SP, 2SP) its own-slot run, E[g][S-1] at CL.  From E's rows (EP
+  // false): E[g][(p0 & ~3) + q] (16-byte copies; the runs p0 + 2j, s0 + 2j,
+  // j <= T, are entries (p0 & 3) + 2j); from the sigma-permuted rows (EP):
+  // the same runs are contiguous, SPP entries each
+  static constexpr int SPP = (T + 1 + 3 + 3) / 4 * 4;
+  static constexpr int SP = EP ? SPP : (2 * T + 4 + 3) / 4 * 4;
   static constexpr int CL = 2 * SP;
   static constexpr int RS = 2 * SP + 4;
   static constexpr int NC = 2 * T + 2;      // pair-0 light-cone tiles (at most)
   static constexpr int NU = (2 * T + 2 + 3 + 3) / 4 * 4;   // their span of E[g][u0 + z], z <= 2T+1
   static constexpr int UOFF = L * RS;       // cone rows follow the rows (one index space)
-  static constexpr int MOFF = UOFF + NC * NU;   // 3 rotating first-firing-class slots (speculative steps)
-  static constexpr int ints = (L * (4 + 1) + MOFF + 4 + 3) / 4 * 4;   // state + g + rows + cone rows + slots
+  static constexpr int MOFF = (UOFF + NC * NU + 1) / 2 * 2;   // 3 rotating 64-bit class masks (speculative steps)
+  static constexpr int ints = (L * (4 + 1) + MOFF + 6 + 3) / 4 * 4;   // state + g + rows + cone rows + masks
   static constexpr size_t bytes = sizeof(int32_t) * (size_t)ints;
 };
 
 
-// Speculative class steps pay once firing classes are rare in a chunk's
-// trapezoid: a speculative iteration (batch test + first-class reduction +
-// apply, two barriers) costs ~3 chain steps (measured), so they
-// are used from the second round on, when the previous round's swaps put
-// fewer than ~1/8 firing pairs per class into an X-pair range (the previous
-// round's count over-estimates this round's).  mode: trap_spec (0 never,
-// 1 this rule, 2 always).  Results are identical either way.
-__device__ __forceinline__ bool spec_round(int32_t mode, int64_t prev_rs, int32_t X, int32_t ncls, int32_t npairs) {
+// Speculative class steps pay only once nearly every chunk's phase is quiet:
+// a pass (every remaining class tested, the first firing class applied) costs
+// a few chain steps, and a phase needs 1 + (firing classes) passes, so busy
+// chunks get slower while quiet ones get faster -- and in the chain of
+// neighbour-synchronised chunks the slow ones pace everybody (measured,
+// DESIGN.md).  So they are used from the second round on, when the previous
+// round's swaps predict f = swaps * X * T / (classes * pairs) < 3/4 firing
+// classes per chunk and phase (the previous round's count over-estimates
+// this round's).  mode: trap_spec (0 never, 1 this rule, 2 always).  Results
+// are identical either way.
+__device__ __forceinline__ bool spec_round(int32_t mode, int64_t prev_rs, int32_t X, int32_t T, int32_t ncls,
+                                           int32_t npairs) {
   if (mode == 2) return true;
   if (mode != 1 || prev_rs < 0) return false;
-  return prev_rs * (int64_t)X * 8 < (int64_t)ncls * npairs;
+  return prev_rs * (int64_t)X * T * 4 < (int64_t)ncls * npairs * 3;
 }
 
 __device__ __forceinline__ int32_t wrap_m(int32_t x, int32_t m) {
@@ -233,15 +239,15 @@ struct TrapChunk {
 
 // One chunk of one phase: stage (state via `src`, E rows from global), replay
 // Tp classes.  Returns the swaps of the owned pairs.
-template <int PPL, int T, typename Src>
+template <int PPL, int T, bool EP, typename Src>
 __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_t k1, int32_t c0, int32_t u0,
                                           const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
                                           int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
                                           bool vec, unsigned long long* tprof,
                                           const int32_t* __restrict__ Ep, int64_t ldp, bool spec, bool pf, int exp = 0,
                                           bool coal = false) {
-  using SM = TrapSmem<PPL, T>;
-  static_assert(T <= 32, "one mask bit per class of a phase");
+  using SM = TrapSmem<PPL, T, EP>;
+  static_assert(T <= 64, "one mask bit per class of a phase");
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
   const bool low = (C.a == 0);
@@ -276,7 +282,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     const int32_t s0 = fx ? u0 : x;
     const int32_t* row = E + (int64_t)g * ld;
     int32_t* dst = s_E + j * RS;
-    if (Ep) {
+    if (EP) {
       // sigma-permuted rows: Ep[g][q] = E[g][2q mod m], so the stride-2 run
       // from column y is the contiguous run from q = sigma(y) = y (m+1)/2
       const int32_t sp = (int32_t)(((int64_t)p0 * ((m + 1) / 2)) % m);
@@ -320,7 +326,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     // that paced the whole chunk chain: config 4 TRAP round 5.5 -> 5.0 ms.)
     if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, aligned || vec);
   }
-  if (Ep && coal && !(exp & 2)) {
+  if (EP && coal && !(exp & 2)) {
     // warp-cooperative copies of the runs of the warp's 32 slots: lane l of
     // copy `ins` moves 16-byte piece P = 32 ins + l of the warp's 64 runs, so
     // one warp instruction covers ~3.5 whole runs (contiguous pieces, ~18
@@ -343,7 +349,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       }
     }
   }
-  if (spec && gt < 3) s_E[SM::MOFF + gt] = 0;
+  if (spec && gt < 6) s_E[SM::MOFF + gt] = 0;
   cp_async_wait_all();
   group_sync(bar_id, GT);
   if (exp & 4) return 0;
@@ -374,12 +380,12 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     // exactly the firing pairs of t* are applied (the pairs of a class are
     // disjoint) and the next pass resumes at t* + 1.  A quiet phase thus
     // costs one parallel pass instead of Tp dependent steps.
-    unsigned int* s_or = reinterpret_cast<unsigned int*>(s_E + SM::MOFF);   // reset before the staging barrier
+    unsigned long long* s_or = reinterpret_cast<unsigned long long*>(s_E + SM::MOFF);   // reset before the staging barrier
     int32_t tc = 0;
     uint32_t it = 0;
     while (tc < Tp) {
       const int32_t tl = min(Tp, tmax + 1);
-      uint32_t mask = 0;
+      unsigned long long mask = 0;
 #pragma unroll 8
       for (int32_t t = tc; t < tl; ++t) {
         const int32_t j1 = (t <= tk) ? b1 + t : c1 - t;
@@ -387,18 +393,20 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
         const int4 A = s_st[j1], B = s_st[j2];
         const int32_t e_bu = s_E[B.z + t * (B.x >> 16)];
         const int32_t e_av = s_E[(k == 0) ? (A.x & 0xffff) * RS + SM::CL : A.z + t * (A.x >> 16)];
-        mask |= (A.y + B.y > e_bu + e_av) ? (1u << t) : 0u;
+        mask |= (A.y + B.y > e_bu + e_av) ? (1ull << t) : 0ull;
       }
-      unsigned int* slot = s_or + (it % 3u);
-      if (gt == 0) s_or[(it + 1) % 3u] = 0u;   // last read two passes ago
-      const uint32_t wor = __reduce_or_sync(0xffffffffu, mask);
+      unsigned long long* slot = s_or + (it % 3u);
+      if (gt == 0) s_or[(it + 1) % 3u] = 0ull;   // last read two passes ago
+      const uint32_t wlo = __reduce_or_sync(0xffffffffu, (uint32_t)mask);
+      const uint32_t whi = (T > 32) ? __reduce_or_sync(0xffffffffu, (uint32_t)(mask >> 32)) : 0u;
+      const unsigned long long wor = ((unsigned long long)whi << 32) | wlo;
       if ((gt & 31) == 0 && wor) atomicOr(slot, wor);
       group_sync(bar_id, GT);
-      const uint32_t all = *slot;
+      const unsigned long long all = *slot;
       ++it;
-      if (all == 0u) break;                    // nothing fires in [tc, Tp): the phase is decided
-      const int32_t ts = __ffs(all) - 1;       // first firing class
-      if ((mask >> ts) & 1u) {                 // apply my pair of class ts (state unchanged since tc)
+      if (all == 0ull) break;                  // nothing fires in [tc, Tp): the phase is decided
+      const int32_t ts = __ffsll((long long)all) - 1;   // first firing class
+      if ((mask >> ts) & 1ull) {               // apply my pair of class ts (state unchanged since tc)
         const int32_t j1 = (ts <= tk) ? b1 + ts : c1 - ts;
         const int32_t j2 = (k == 0) ? Lc - 1 : ((ts >= k) ? b2 + ts : c2 - ts);
         const int4 fA = s_st[j1], fB = s_st[j2];
@@ -449,10 +457,10 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
   return mysw;
 }
 
-template <int PPL, int T, bool CLU>
+template <int PPL, int T, bool CLU, bool EP>
 __global__ void __launch_bounds__(256, 1)
 k_ls_trap(const TrapParams p) {
-  using SM = TrapSmem<PPL, T>;
+  using SM = TrapSmem<PPL, T, EP>;
   constexpr int L = SM::L, X = SM::X;
   extern __shared__ __align__(16) int32_t sm[];
   constexpr int GT = X;                        // threads per chunk group (PPL warps)
@@ -528,7 +536,7 @@ k_ls_trap(const TrapParams p) {
   uint32_t qph = 0;      // grid mode: phases completed
   int64_t prev_rs = -1;   // swaps of the previous round (-1: none yet)
   for (;;) {
-    const bool spec = spec_round(p.spec, prev_rs, X, ncls, K + 1);
+    const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1);
     if (!CLU && blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
@@ -547,7 +555,7 @@ k_ls_trap(const TrapParams p) {
         if (have) {
           if (CLU) {
             const int2* rr = rep + cur * S;
-            mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
+            mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { const int2 v = rr[x]; g = v.x; d = v.y; el = -1; },
                                        s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
           } else {
@@ -570,7 +578,7 @@ k_ls_trap(const TrapParams p) {
               }
               group_sync(1 + grp, GT);
             }
-            mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
+            mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) {
                                          const int4 v = __ldcg(sc + x); g = v.x; d = v.y; el = v.z;
                                        },
@@ -708,9 +716,9 @@ k_ls_trap(const TrapParams p) {
 
 int32_t ls_trap_min_S() { return 256; }
 
-template <int PPL, int T>
-static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
-  using SM = TrapSmem<PPL, T>;
+template <int PPL, int T, bool EP>
+static pm_status_t launch_trap_ep(TrapParams& hp, cudaStream_t st) {
+  using SM = TrapSmem<PPL, T, EP>;
   constexpr int X = SM::X;
   static_assert(X > 2 * T + 1, "chunk must own more than T pairs");
   int dev = 0, nsm = 0, optin = 0;
@@ -743,7 +751,7 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
     if (nblk > 16) return PM_ERR_UNSUPPORTED;
     const size_t smem = SM::bytes * cpc_cl + rep_bytes;
     const int threads = 32 * gsz * cpc_cl;
-    auto fn = k_ls_trap<PPL, T, true>;
+    auto fn = k_ls_trap<PPL, T, true, EP>;
     PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     if (nblk > 8) PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     cudaLaunchConfig_t cfg = {};
@@ -776,7 +784,7 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   if (cpc > max_cpc) cpc = max_cpc;
   const size_t smem = SM::bytes * cpc;
   const int threads = 32 * gsz * cpc;
-  auto fn = k_ls_trap<PPL, T, false>;
+  auto fn = k_ls_trap<PPL, T, false, EP>;
   PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
@@ -787,6 +795,14 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
   PM_CUDA_TRY(cudaLaunchCooperativeKernel((const void*)fn, dim3(grid), dim3(threads), args, smem, st));
   note_launch();
   return PM_OK;
+}
+
+// The staging layout depends on whether the runs come from the sigma-permuted
+// copy (EP: contiguous runs, half the shared memory per tile) or from E.
+template <int PPL, int T>
+static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
+  if (hp.Ep) return launch_trap_ep<PPL, T, true>(hp, st);
+  return launch_trap_ep<PPL, T, false>(hp, st);   // PM_ERR_UNSUPPORTED if its layout exceeds shared memory
 }
 
 pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
@@ -848,13 +864,17 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
     case 3: return launch_trap<4, 16>(hp, st);
     case 4: return launch_trap<4, 8>(hp, st);
     case 5: return launch_trap<4, 32>(hp, st);
+    case 6: return launch_trap<6, 48>(hp, st);
     default:
-      // measured: 64-pair ranges x 16 classes while E is
-      // L2-resident; 128 x 32 from HBM while its 128-thread chunks fit one
-      // pass of the grid (config 4: 76.3 -> 67.9 ms; config 5 stays at
-      // 64 x 16: 1.21 vs 1.32 s)
-      if ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) return launch_trap<4, 32>(hp, st);
-      return launch_trap<2, 16>(hp, st);
+      // measured (whole search, configs 1/2/3/4): 128-pair ranges
+      // x 32 classes 0.338/1.049/6.14/36.6 ms, 64 x 16 0.353/1.172/7.73/54.9,
+      // 192 x 48 0.353/1.107/6.20/34.5 -- so 192 x 48 once E is beyond L2
+      // (it needs the sigma-permuted copy's compact staging), 128 x 32 below;
+      // from E's own rows (E > 2 GiB, config 5) 64 x 16 (round 1: 1.21 vs
+      // 1.32 s for 128 x 32)
+      if (!hp.Ep) return launch_trap<2, 16>(hp, st);
+      if ((int64_t)S * ldE * 4 > (96ll << 20)) return launch_trap<6, 48>(hp, st);
+      return launch_trap<4, 32>(hp, st);
   }
 }
 
@@ -964,10 +984,10 @@ __device__ __forceinline__ bool sys_barrier_arrive_wait(const TrapMultiParams& p
   return wait_ge_sys(p, r, p.rk[r].xbar, target);
 }
 
-template <int PPL, int T>
+template <int PPL, int T, bool EP>
 __global__ void __launch_bounds__(256, 1)
 k_ls_trap_mr(const TrapMultiParams p) {
-  using SM = TrapSmem<PPL, T>;
+  using SM = TrapSmem<PPL, T, EP>;
   constexpr int L = SM::L, X = SM::X, GT = X;
   extern __shared__ __align__(16) int32_t sm[];
   const int cpc = blockDim.x / GT;
@@ -1011,7 +1031,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
   unsigned int xtarget = 0;
   int64_t prev_rs = -1;
   while (ok) {
-    const bool spec = spec_round(p.spec, prev_rs, X, ncls, K + 1);
+    const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1);
     if (leader) me.rtot[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls && ok; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
@@ -1039,7 +1059,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
           C.K = K; C.m = m; C.Tp = Tp;
           const int32_t* __restrict__ rc = me.rbuf[bi];
           const int32_t* __restrict__ dc = me.dbuf[bi];
-          mysw += trap_chunk<PPL, T>(C, k0, k1, c0, u0, E, ld, S,
+          mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
                                      [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { g = __ldcg(rc + x); d = __ldcg(dc + x); el = -1; },
                                      s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp, spec, p.prefetch, 0, p.coal);
           // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
@@ -1184,12 +1204,12 @@ static void trap_ws_layout(void* ws, int32_t S, int32_t* perm, const int32_t* E,
 size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((size_t)S / 2 + 16); }
 
 // Launch `nloc` ranks [rank0, rank0 + nloc) of a world on the current device.
-template <int PPL, int T>
+template <int PPL, int T, bool EP>
 static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE,
                                      int32_t S, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
                                      int32_t max_log, cudaStream_t st, int32_t* handoff, int32_t sparse_T,
                                      int64_t ldp) {
-  using SM = TrapSmem<PPL, T>;
+  using SM = TrapSmem<PPL, T, EP>;
   if (S < ls_trap_min_S() || (S & 1) || world < 1 || world > kMaxRanks || nloc < 1) return PM_ERR_UNSUPPORTED;
   int dev = 0, nsm = 0, optin = 0;
   PM_CUDA_TRY(cudaGetDevice(&dev));
@@ -1219,7 +1239,7 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   if (cpc > max_cpc) cpc = max_cpc;
   const size_t smem = SM::bytes * cpc;
   const int threads = SM::X * cpc;
-  auto fn = k_ls_trap_mr<PPL, T>;
+  auto fn = k_ls_trap_mr<PPL, T, EP>;
   PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
@@ -1244,11 +1264,16 @@ static int32_t trap_multi_variant(int32_t S, int64_t ldE) {
 pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
                            int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                            cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0, int64_t ldp = 0) {
+  const bool ep = ranks[rank0].Ep != nullptr;
   if (trap_multi_variant(S, ldE) == 5)
-    return launch_trap_multi<4, 32>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log,
-                                    st, handoff, sparse_T, ldp);
-  return launch_trap_multi<2, 16>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
-                                  handoff, sparse_T, ldp);
+    return ep ? launch_trap_multi<4, 32, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                               max_log, st, handoff, sparse_T, ldp)
+              : launch_trap_multi<4, 32, false>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                                max_log, st, handoff, sparse_T, ldp);
+  return ep ? launch_trap_multi<2, 16, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                             max_log, st, handoff, sparse_T, ldp)
+            : launch_trap_multi<2, 16, false>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                              max_log, st, handoff, sparse_T, ldp);
 }
 
 
