@@ -218,10 +218,24 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   }
   const int32_t sparse_T = (method == PM_LS_CLASS || method == PM_LS_WINDOW || method == PM_LS_TRAP)
                                ? ls_sparse_threshold(S, method) : 0;
+  // TRAP's sigma-permuted copy of E lives through the sparse rounds too: their
+  // first (full) scan streams its rows instead of gathering from E
+  ScopedScratch ep(st);
+  int64_t ldp = 0;
+  if (method == PM_LS_TRAP) {
+    PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
+    int32_t* Ep = nullptr;
+    const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+    ep.p = Ep;
+    if (se != PM_OK) return se;
+  }
   SparseRun sr;
+  ScopedScratch sps(st);
   if (sparse_T > 0) {
-    const pm_status_t s = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &sr);
+    const pm_status_t s = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &sr, 0,
+                                         ep.as<int32_t>(), ldp);
     if (s != PM_OK) return s;
+    sps.p = sr.scratch;   // freed here on an error path; sparse_launch frees it otherwise
   }
   pm_status_t s;
   switch (method) {
@@ -229,7 +243,8 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
       s = run_class(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
       break;
     case PM_LS_TRAP:
-      s = run_trap(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
+      s = run_trap(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T,
+                   ep.as<int32_t>(), ldp);
       break;
     case PM_LS_WINDOW:
       s = run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);
@@ -248,10 +263,8 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
       return PM_ERR_UNSUPPORTED;
   }
   if (sparse_T > 0) {
-    if (s != PM_OK) {
-      cudaFreeAsync(sr.scratch, st);
-      return s;
-    }
+    if (s != PM_OK) return s;
+    sps.p = nullptr;
     return sparse_launch(&sr, st);
   }
   return s;

@@ -56,24 +56,131 @@ __global__ void k_sp_begin(SpParams* p, cudaGraphConditionalHandle h) {
     const unsigned cont = (p->out->status == PM_OK && p->pending) ? 1u : 0u;
     p->pending = 0;
     p->nd_prev = -1;                             // the dense stage's swaps are not listed: full scan
+#ifdef PM_LS_PROFILE
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (p->max_log >= 1024) p->per_round[1023] = (int64_t)t;   // sparse stage start (tools/sp_rounds.py)
+#endif
     cudaGraphSetConditional(h, cont);
+  }
+}
+
+// Full scan from the sigma-permuted copy Ep[t][q] = E[t][2q mod m] (TRAP
+// keeps it for the sparse rounds).  For a regular slot y with tile r[y], its
+// partner in class c is (2c+1-y) mod m, whose sigma-position is
+// (c + (m+1)/2 - sigma(y)) mod m: consecutive classes read consecutive
+// entries of row r[y].  So with w_y(c) = E[r[y]][partner_c(y)] - d[y], the
+// pair (u, v) of class c fires iff w_u(c) + w_v(c) < 0 (line 5), and a tile
+// of kScanU slots x kScanB classes needs the streams of its slots and of the
+// kScanU + 2 kScanB - 2 partner slots over those classes -- coalesced rows
+// instead of two scattered gathers per pair.  The fixed point u0 of each
+// class and slot S-1 (even S) are tested separately.
+constexpr int kScanU = 256, kScanB = 32, kScanVB = kScanU + 2 * kScanB;
+constexpr size_t kScanSmem = sizeof(int32_t) * (size_t)(kScanU + kScanVB) * kScanB;
+
+__device__ __forceinline__ void scan_full_ep(const SpParams* __restrict__ p, int32_t stamp, int32_t* sm) {
+  const Classes cl(p->S);
+  const int32_t m = cl.m, H = cl.half, S = p->S;
+  const int32_t* __restrict__ r = p->r;
+  const int32_t* __restrict__ d = p->d;
+  const int32_t* __restrict__ Ep = p->Ep;
+  const int64_t ldp = p->ldp;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+  int32_t* wA = sm;                      // [kScanU][kScanB]
+  int32_t* wB = sm + kScanU * kScanB;    // [kScanVB][kScanB]
+  const int32_t nU = (m + kScanU - 1) / kScanU, nC = (m + kScanB - 1) / kScanB;
+  for (int32_t tile = blockIdx.x; tile < nU * nC; tile += gridDim.x) {
+    const int32_t x0 = (tile % nU) * kScanU, c0 = (tile / nU) * kScanB;
+    int32_t vbase = (int32_t)(((int64_t)2 * c0 + 1 - x0 - (kScanU - 1)) % m);
+    vbase = vbase < 0 ? vbase + m : vbase;
+    const int32_t c = c0 + lane;
+    // rows in groups of 32 per warp: lane l fetches row l's tile, d and start
+    // position (coalesced), then the warp streams the 32 rows' class runs
+    // (one 128-byte load each, all in flight together)
+    constexpr int NG = (kScanU + kScanVB) / 32;
+    for (int32_t grp = warp; grp < NG; grp += nwarp) {
+      const int32_t row = grp * 32 + lane;
+      int32_t y;
+      bool ok = true;
+      if (row < kScanU) {
+        y = x0 + row;
+        ok = y < m;
+      } else {
+        y = (vbase + (row - kScanU)) % m;   // (m may be below kScanVB: rows then repeat)
+      }
+      int32_t t = 0, dy = 0, q = 0;
+      if (ok) {
+        t = __ldg(r + y);
+        dy = __ldg(d + y);
+        q = (int32_t)(((int64_t)c0 + H - (int64_t)y * H % m) % m);   // sigma-position of class c0's partner
+        q = q < 0 ? q + m : q;
+      }
+      int32_t val[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const int32_t ti = __shfl_sync(0xffffffffu, t, i);
+        const int32_t qi = __shfl_sync(0xffffffffu, q, i);
+        val[i] = __ldg(Ep + (int64_t)ti * ldp + qi + lane);   // qi + lane < m + 32 <= ldp (cyclic copy)
+      }
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const int32_t di = __shfl_sync(0xffffffffu, dy, i);
+        const int32_t oi = __shfl_sync(0xffffffffu, ok ? 1 : 0, i);
+        const int32_t ri = grp * 32 + i;
+        int32_t* dst = ri < kScanU ? wA + ri * kScanB : wB + (ri - kScanU) * kScanB;
+        dst[lane] = (oi && c < m) ? val[i] - di : 0;
+      }
+    }
+    __syncthreads();
+    if (c < m) {
+      int32_t u0 = c + H;
+      u0 = u0 >= m ? u0 - m : u0;
+      for (int32_t ur = warp; ur < kScanU; ur += nwarp) {
+        const int32_t u = x0 + ur;
+        if (u >= m || u == u0) continue;
+        int32_t v = 2 * c + 1 - u;
+        v = v < 0 ? v + m : (v >= m ? v - m : v);
+        int32_t vr = v - vbase;
+        vr = vr < 0 ? vr + m : vr;
+        if ((int64_t)wA[ur * kScanB + lane] + wB[vr * kScanB + lane] < 0) p->flags[c] = stamp;
+      }
+    }
+    __syncthreads();
+  }
+  if (S % 2 == 0) {   // the pairs (u0(c), S-1)
+    const int32_t* __restrict__ E = p->E;
+    const int64_t ld = p->ldE;
+    for (int32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < m; c += gridDim.x * blockDim.x) {
+      int32_t u0 = c + H;
+      u0 = u0 >= m ? u0 - m : u0;
+      const int32_t a = __ldg(r + u0), b = __ldg(r + S - 1);
+      if ((int64_t)__ldg(d + u0) + __ldg(d + S - 1) >
+          (int64_t)__ldg(E + (int64_t)b * ld + u0) + __ldg(E + (int64_t)a * ld + (S - 1)))
+        p->flags[c] = stamp;
+    }
   }
 }
 
 // Stamp every class that has a firing pair on the round's start state.  A
 // pair whose slots were not swapped during the previous round did not fire
 // then on the same values, so after a sparse round only the pairs of the
-// slots it swapped (dprev) are tested; after the dense stage, all pairs.
+// slots it swapped (dprev) are tested; after the dense stage, all pairs
+// (streamed from Ep when TRAP left it, else gathered from E).
 __global__ void __launch_bounds__(256) k_sp_scan(const SpParams* __restrict__ p) {
+  extern __shared__ __align__(16) int32_t sm_scan[];
   if (p->out->status != PM_OK) return;
   if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(p->launches, 1ull);
   const Classes cl(p->S);
   const int32_t stamp = (int32_t)p->out->rounds + 1;
+  const int32_t ndp = p->nd_prev;
+  if (ndp < 0 && p->Ep) {
+    scan_full_ep(p, stamp, sm_scan);
+    return;
+  }
   const int32_t* __restrict__ E = p->E;
   const int32_t* __restrict__ r = p->r;
   const int32_t* __restrict__ d = p->d;
   const int64_t ld = p->ldE;
-  const int32_t ndp = p->nd_prev;
   const int64_t total = ndp >= 0 ? (int64_t)cl.ncls * ndp : (int64_t)cl.ncls * cl.npairs;
   const int32_t per = ndp >= 0 ? ndp : cl.npairs;
   for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
@@ -493,7 +600,10 @@ static cudaError_t build_sparse_graph(int32_t S, bool use_smem, bool cluster, Sp
   if ((e = cudaStreamEndCapture(cs, &captured)) != cudaSuccess) return e;
   if ((e = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed)) != cudaSuccess)
     return e;
-  k_sp_scan<<<scan_blocks(S), 256, 0, cs>>>(out.dparams);
+  if ((e = cudaFuncSetAttribute(k_sp_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kScanSmem)) !=
+      cudaSuccess)
+    return e;
+  k_sp_scan<<<scan_blocks(S), 256, kScanSmem, cs>>>(out.dparams);
   if (cluster) {
     if ((e = launch_cwalk(out.dparams, h, S, use_smem, cs)) != cudaSuccess) {
       cudaStreamEndCapture(cs, &captured);
@@ -538,7 +648,7 @@ int32_t ls_sparse_threshold(int32_t S, int32_t dense_method) {
 
 pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                            LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                           SparseRun* run, int32_t pending0) {
+                           SparseRun* run, int32_t pending0, const int32_t* Ep, int64_t ldp) {
   int dev = 0, optin = 0;
   PM_CUDA_TRY(cudaGetDevice(&dev));
   PM_CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
@@ -582,6 +692,8 @@ pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* pe
   hp.dprev = hp.flist + (cl.ncls + 1);
   hp.gbuf = use_smem ? nullptr : hp.dprev + S;
   hp.nd_prev = -1;
+  hp.Ep = (Ep && S >= 2 && ldp >= (int64_t)Classes(S).m + 32) ? Ep : nullptr;
+  hp.ldp = ldp;
   hp.S = S; hp.max_rounds = max_rounds; hp.max_log = max_log;
   hp.pending = pending0; hp.use_smem = use_smem ? 1 : 0;
   hp.out = dev_out; hp.per_round = dev_per_round;

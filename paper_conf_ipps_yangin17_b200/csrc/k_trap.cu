@@ -797,6 +797,23 @@ static pm_status_t launch_trap_ep(TrapParams& hp, cudaStream_t st) {
   return PM_OK;
 }
 
+// sigma-permuted copy of E: up to E = 2 GiB (trap_ep 1, measured: config 2
+// 1.25 -> 1.18 ms, config 4 67.4 -> 62.3 ms; config 5 1.09 -> 1.25 s --
+// building the 16 GiB copy costs more than it saves), always (2), never (0).
+// The runs become contiguous: dense sectors instead of stride-2 ones.
+pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
+                                 int64_t* ldp) {
+  *Ep = nullptr;
+  *ldp = 0;
+  const int32_t ep_mode = knob("trap_ep", 1);
+  if (ep_mode == 0 || (ep_mode == 1 && (int64_t)S * ldE * 4 > (2ll << 30))) return PM_OK;
+  const int32_t m = S - 1, ext = 48;
+  *ldp = ((int64_t)m + ext + 31) / 32 * 32;
+  PM_CUDA_TRY(pm::scratch_alloc(Ep, sizeof(int32_t) * (size_t)S * (size_t)*ldp, st));
+  PM_CUDA_TRY(launch_permute_cols(E, ldE, *Ep, *ldp, S, m, ext, st));
+  return PM_OK;
+}
+
 // The staging layout depends on whether the runs come from the sigma-permuted
 // copy (EP: contiguous runs, half the shared memory per tile) or from E.
 template <int PPL, int T>
@@ -807,9 +824,9 @@ static pm_status_t launch_trap(TrapParams& hp, cudaStream_t st) {
 
 pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                      LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                     int32_t* handoff, int32_t sparse_T) {
+                     int32_t* handoff, int32_t sparse_T, const int32_t* Ep_in, int64_t ldp_in) {
   if (S < ls_trap_min_S() || (S & 1)) return PM_ERR_UNSUPPORTED;
-  PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
+  // (run_local_search checks the permutation before building Ep)
   // scratch: 3 round counters, barrier counter, chunk flags [S/2], then the
   // three generations of packed slot states (int4 [S] each)
   const size_t n = (size_t)S;
@@ -843,15 +860,17 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   // from HBM)
   // (measured: config 2 1.25 -> 1.18 ms, config 4 67.4 -> 62.3 ms; config 5
   // 1.09 -> 1.25 s -- building the 16 GiB copy costs more than it saves)
-  const int32_t ep_mode = knob("trap_ep", 1);   // 0 off, 1 up to E = 2 GiB, 2 always
-  if (ep_mode == 2 || ((int64_t)S * ldE * 4 <= (2ll << 30) && ep_mode == 1)) {
-    const int32_t m = S - 1, ext = 48;   // >= SPP + 4 for every T used
-    const int64_t ldp = ((int64_t)m + ext + 31) / 32 * 32;
-    PM_CUDA_TRY(pm::scratch_alloc(&ep.p, sizeof(int32_t) * (size_t)S * (size_t)ldp, st));
-    PM_CUDA_TRY(launch_permute_cols(E, ldE, ep.as<int32_t>(), ldp, S, m, ext, st));
-    hp.Ep = ep.as<int32_t>(); hp.ldp = ldp;
-    if ((int64_t)S * ldp >= (1ll << 31)) hp.coal = 0;   // int32 element offsets
+  if (Ep_in) {
+    hp.Ep = Ep_in; hp.ldp = ldp_in;
+  } else {
+    int32_t* Ep = nullptr;
+    int64_t ldp = 0;
+    const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+    ep.p = Ep;
+    if (se != PM_OK) return se;
+    hp.Ep = Ep; hp.ldp = ldp;
   }
+  if (hp.Ep && (int64_t)S * hp.ldp >= (1ll << 31)) hp.coal = 0;   // int32 element offsets
   // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
   // used runs win (config 4: 5.0 vs 10.8 us)
@@ -1276,20 +1295,6 @@ pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_
                                               max_log, st, handoff, sparse_T, ldp);
 }
 
-
-// sigma-permuted copy of E up to E = 2 GiB (as run_trap); NULL else.
-static pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
-                                 int64_t* ldp) {
-  *Ep = nullptr;
-  *ldp = 0;
-  const int32_t ep_mode = knob("trap_ep", 1);
-  if (ep_mode == 0 || (ep_mode == 1 && (int64_t)S * ldE * 4 > (2ll << 30))) return PM_OK;
-  const int32_t m = S - 1, ext = 48;
-  *ldp = ((int64_t)m + ext + 31) / 32 * 32;
-  PM_CUDA_TRY(pm::scratch_alloc(Ep, sizeof(int32_t) * (size_t)S * (size_t)*ldp, st));
-  PM_CUDA_TRY(launch_permute_cols(E, ldE, *Ep, *ldp, S, m, ext, st));
-  return PM_OK;
-}
 
 // Can the multi-rank kernel take (S, world)?  Checked before anything is
 // enqueued (pm.h: arguments are validated before any launch).

@@ -149,6 +149,8 @@ struct SpParams {
   int32_t use_smem;
   int32_t nd_prev;             // slots swapped in the previous sparse round (-1: unknown)
   int32_t* dprev;              // [S] their list
+  const int32_t* Ep;           // sigma-permuted copy of E (or NULL): the full scan streams its rows
+  int64_t ldp;
   LsResult* out;
   int64_t* per_round;
   unsigned long long* launches;   // device-side launch counter (graph kernels)
@@ -170,7 +172,7 @@ int32_t ls_sparse_threshold(int32_t S, int32_t dense_method);
 // has checked that perm is a bijection.
 pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                            LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                           SparseRun* run, int32_t pending0 = 0);
+                           SparseRun* run, int32_t pending0 = 0, const int32_t* Ep = nullptr, int64_t ldp = 0);
 // dev_out->status = PM_ERR_NOT_PERMUTATION unless perm is a bijection of [0, S).
 cudaError_t launch_perm_check(const int32_t* perm, int32_t S, LsResult* dev_out, cudaStream_t st);
 // ... and the sparse-round graph (after it).
@@ -184,7 +186,11 @@ int64_t device_launch_total();
 int32_t ls_trap_min_S();
 pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                      LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                     int32_t* handoff, int32_t sparse_T);
+                     int32_t* handoff, int32_t sparse_T, const int32_t* Ep = nullptr, int64_t ldp = 0);
+// The sigma-permuted copy Ep[t][q] = E[t][2q mod m] (q < m + 48, cyclic) that
+// TRAP stages from while E <= 2 GiB (trap_ep), or NULL: allocated from the
+// scratch pool on st; the caller frees it.
+pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep, int64_t* ldp);
 
 // Multi-rank TRAP (k_trap.cu).
 struct TrapRank;

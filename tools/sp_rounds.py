@@ -31,7 +31,7 @@ for r in range(rounds):
     if full[832 + r] == 0:
         print(f"round {r}: swaps={full[r]} (dense stage)")
         continue
-    gap = (full[832 + r] - prev_end) if prev_end else 0
+    gap = (full[832 + r] - prev_end) if prev_end else (full[832 + r] - full[1023] if full[1023] else 0)
     prev_end = full[896 + r]
     print(f"round {r}: swaps={full[r]:6d} walk={dur/1e3:8.1f} us gap-before(scan+launch)={gap/1e3:7.1f} us "
           f"windows={full[576 + r]} applies={full[640 + r]} dirty_end={full[704 + r]} stamped={full[768 + r]} "
