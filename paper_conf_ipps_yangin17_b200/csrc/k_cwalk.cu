@@ -80,7 +80,8 @@ __global__ void __launch_bounds__(cw::kThreads, 1) k_sp_cwalk(SpParams* p, cudaG
   const int rank = (int)cluster.block_rank();
   extern __shared__ __align__(16) int32_t smem[];
   __shared__ CwMail s_mail[2][C];
-  __shared__ int32_t s_fl[cw::kFl];
+  constexpr int kFlC = C > 8 ? cw::kFl / 2 : cw::kFl;
+  __shared__ int32_t s_fl[kFlC];
   __shared__ int32_t s_nd, s_lmin[2], s_cnt[2], s_red[32];
   const int32_t S = p->S;
   const Classes cl(S);
@@ -120,7 +121,7 @@ __global__ void __launch_bounds__(cw::kThreads, 1) k_sp_cwalk(SpParams* p, cudaG
   int32_t pos = 0;
   const int32_t nf = cw_block_scan(cnt, pos, s_red);
   const int32_t* FL;
-  if (nf <= cw::kFl) {
+  if (nf <= kFlC) {
     for (int32_t c = c0; c < c1; ++c)
       if (p->flags[c] == stamp) s_fl[pos++] = c;
     FL = s_fl;
@@ -446,35 +447,51 @@ __global__ void __launch_bounds__(cw::kThreads, 1) k_sp_cwalk(SpParams* p, cudaG
 namespace pm {
 
 namespace {
-constexpr int kCwCluster = 8;                    // portable cluster size
-constexpr size_t kCwStaticSmem = sizeof(CwMail) * 2 * kCwCluster + sizeof(int32_t) * (cw::kFl + 40);
+// cluster sizes: 8 (portable) or 16 (non-portable; tuning ls_cwalk_c)
+template <int C>
+constexpr size_t cw_static_smem() {
+  return sizeof(CwMail) * 2 * C + sizeof(int32_t) * ((C > 8 ? cw::kFl / 2 : cw::kFl) + 40);
+}
 }  // namespace
 
-bool cwalk_smem_ok(int32_t S, int optin) { return cwalk_state_bytes(S) + kCwStaticSmem + 1024 <= (size_t)optin; }
-size_t cwalk_gbuf_bytes(int32_t S) { return cwalk_state_bytes(S) * kCwCluster; }
+// 16 CTAs by default (measured: config 4 whole search 29.4 -> 28.5 ms; the
+// windows are bound by the gathers of the cluster's SMs), 8 by tuning
+int32_t cwalk_cluster() { return knob("ls_cwalk_c", 16) >= 16 ? 16 : 8; }
 
-// One cluster of kCwCluster CTAs (enqueued on st, e.g. while capturing the
-// sparse-round graph).
-cudaError_t launch_cwalk(SpParams* p, cudaGraphConditionalHandle h, int32_t S, bool smem, cudaStream_t st) {
+bool cwalk_smem_ok(int32_t S, int optin) {
+  const size_t st = cwalk_cluster() == 16 ? cw_static_smem<16>() : cw_static_smem<8>();
+  return cwalk_state_bytes(S) + st + 1024 <= (size_t)optin;
+}
+size_t cwalk_gbuf_bytes(int32_t S) { return cwalk_state_bytes(S) * cwalk_cluster(); }
+
+template <int C>
+static cudaError_t launch_cwalk_c(SpParams* p, cudaGraphConditionalHandle h, int32_t S, bool smem, cudaStream_t st) {
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(kCwCluster, 1, 1);
+  cfg.gridDim = dim3(C, 1, 1);
   cfg.blockDim = dim3(cw::kThreads, 1, 1);
   cfg.dynamicSmemBytes = smem ? cwalk_state_bytes(S) : 0;
   cfg.stream = st;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeClusterDimension;
-  at[0].val.clusterDim.x = kCwCluster;
+  at[0].val.clusterDim.x = C;
   at[0].val.clusterDim.y = 1;
   at[0].val.clusterDim.z = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  if (smem) {
-    cudaError_t e = cudaFuncSetAttribute(k_sp_cwalk<kCwCluster, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)cfg.dynamicSmemBytes);
-    if (e != cudaSuccess) return e;
-    return cudaLaunchKernelEx(&cfg, k_sp_cwalk<kCwCluster, true>, p, h);
-  }
-  return cudaLaunchKernelEx(&cfg, k_sp_cwalk<kCwCluster, false>, p, h);
+  auto fn = smem ? k_sp_cwalk<C, true> : k_sp_cwalk<C, false>;
+  cudaError_t e;
+  if (C > 8 && (e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1)) != cudaSuccess)
+    return e;
+  if (smem && (e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)cfg.dynamicSmemBytes)) != cudaSuccess)
+    return e;
+  return cudaLaunchKernelEx(&cfg, fn, p, h);
+}
+
+// One cluster of the walk's CTAs (enqueued on st, e.g. while capturing the
+// sparse-round graph).
+cudaError_t launch_cwalk(SpParams* p, cudaGraphConditionalHandle h, int32_t S, bool smem, cudaStream_t st) {
+  return cwalk_cluster() == 16 ? launch_cwalk_c<16>(p, h, S, smem, st) : launch_cwalk_c<8>(p, h, S, smem, st);
 }
 
 }  // namespace pm

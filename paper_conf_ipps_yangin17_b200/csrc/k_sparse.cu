@@ -557,7 +557,7 @@ struct SpGraph {
 
 // Per host thread and bounded, as the CLASS graph cache (k_search.cu).
 constexpr size_t kSpCacheMax = 64;
-static thread_local std::map<std::tuple<int, int32_t, cudaStream_t, bool, bool>, SpGraph> g_sp_graphs;
+static thread_local std::map<std::tuple<int, int32_t, cudaStream_t, bool, bool, int32_t>, SpGraph> g_sp_graphs;
 
 static int scan_blocks(int32_t S) {
   const int64_t total = (int64_t)Classes(S).ncls * Classes(S).npairs;
@@ -661,7 +661,7 @@ pm_status_t sparse_prepare(const int32_t* E, int64_t ldE, int32_t S, int32_t* pe
                         !knob("ls_sparse_gmem", 0);
   SpGraph sg;
   {
-    auto key = std::make_tuple(dev, S, st, use_smem, cluster);
+    auto key = std::make_tuple(dev, S, st, use_smem, cluster, cluster ? cwalk_cluster() : 1);
     auto it = g_sp_graphs.find(key);
     if (it == g_sp_graphs.end() && g_sp_graphs.size() >= kSpCacheMax) {
       PM_CUDA_TRY(cudaDeviceSynchronize());

@@ -46,16 +46,32 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 // [pos, pos + K + 4) can be read without wrapping.
 __global__ void k_permute_cols(const int32_t* __restrict__ E, int64_t ld, int32_t* __restrict__ Ep, int64_t ldp,
                                int32_t S, int32_t m, int32_t ext) {
+  // rows along y (grid-stride), four consecutive outputs per thread: the
+  // inputs of a warp are 256 consecutive even (or odd) columns of the row,
+  // so every sector is read from DRAM once (its other half by the other
+  // half of the row, from L2) and the outputs are written as 16-byte stores
   const int32_t w = m + ext;
-  const int64_t total = (int64_t)S * w;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t t = i / w;
-    const int32_t orig = (int32_t)(i - t * w);
-    int32_t pos = orig;
-    while (pos >= m) pos -= m;
-    int32_t q = 2 * pos;
-    if (q >= m) q -= m;
-    Ep[t * ldp + orig] = __ldg(E + t * ld + q);
+  const int32_t q0 = 4 * (blockIdx.x * blockDim.x + threadIdx.x);
+  if (q0 >= w) return;
+  const bool vec4 = (ldp % 4 == 0) && ((reinterpret_cast<uintptr_t>(Ep) & 15) == 0);
+  for (int64_t t = blockIdx.y; t < S; t += gridDim.y) {
+    const int32_t* __restrict__ row = E + t * ld;
+    int32_t v[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      int32_t pos = q0 + i;
+      if (pos >= w) { v[i] = 0; continue; }
+      while (pos >= m) pos -= m;
+      int32_t q = 2 * pos;
+      if (q >= m) q -= m;
+      v[i] = __ldg(row + q);
+    }
+    int32_t* dst = Ep + t * ldp + q0;
+    if (vec4 && q0 + 4 <= w) {
+      *reinterpret_cast<int4*>(dst) = make_int4(v[0], v[1], v[2], v[3]);
+    } else {
+      for (int i = 0; i < 4 && q0 + i < w; ++i) dst[i] = v[i];
+    }
   }
 }
 
@@ -454,11 +470,9 @@ int32_t ls_window_max_S() { return 2048; }
 
 cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int64_t ldp, int32_t S, int32_t m,
                                 int32_t ext, cudaStream_t st) {
-  const int64_t total = (int64_t)S * (m + ext);
-  int64_t blocks = (total + 255) / 256;
-  if (blocks > 148 * 8) blocks = 148 * 8;
-  if (blocks < 1) blocks = 1;
-  k_permute_cols<<<(unsigned)blocks, 256, 0, st>>>(E, ldE, Ep, ldp, S, m, ext);
+  const int32_t bx = (m + ext + 4 * 256 - 1) / (4 * 256);
+  const int32_t by = S < 65535 ? S : 65535;
+  k_permute_cols<<<dim3(bx, by), 256, 0, st>>>(E, ldE, Ep, ldp, S, m, ext);
   note_launch();
   return cudaGetLastError();
 }

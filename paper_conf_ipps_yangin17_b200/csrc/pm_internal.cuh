@@ -162,6 +162,7 @@ struct SparseRun {
 };
 // The walk on a thread-block cluster (k_cwalk.cu).
 bool cwalk_smem_ok(int32_t S, int optin);
+int32_t cwalk_cluster();   // CTAs of the walk's cluster (8, or 16 by tuning)
 size_t cwalk_gbuf_bytes(int32_t S);
 cudaError_t launch_cwalk(SpParams* p, cudaGraphConditionalHandle h, int32_t S, bool smem, cudaStream_t st);
 // Swap-count threshold at which the dense stage (WINDOW / CLASS) hands over

@@ -510,6 +510,15 @@ def test_walk_all_rounds_parity(fam, N, M, C):
     _check_ls(oracle_E(fam, N, M, C), "walk")
 
 
+@pytest.mark.parametrize("C", [8, 16])
+@pytest.mark.parametrize("N,M,C_img,fam", [(512, 16, 3, "smooth"), (1440, 32, 1, "noise"), (128, 8, 3, "ties")])
+def test_walk_cluster_sizes(C, N, M, C_img, fam):
+    # the cluster walk on 8 (portable) or 16 (non-portable) CTAs
+    pm.tuning_set("ls_cwalk_c", C)
+    pm.tuning_set("ls_cwalk", 1)
+    _check_ls(oracle_E(fam, N, M, C_img), "walk")
+
+
 def test_walk_mailbox_overflow_falls_back_exactly():
     # T = I with the tiles of 63 pairs of the first colour class exchanged: from
     # the identity all 63 fire in that class, more than one CTA's mailbox holds

@@ -8,7 +8,7 @@ _MAP = {"PM_TRAP_V": "trap_variant", "PM_TRAP_W": "trap_W", "PM_TRAP_CLUSTER": "
         "PM_TRAP_EP": "trap_ep", "PM_TRAP_VEC": "trap_vec", "PM_TRAP_SPEC": "trap_spec",
         "PM_TRAP_PREFETCH": "trap_prefetch", "PM_TRAP_COAL": "trap_coal", "PM_TRAP_EXP": "trap_exp",
         "PM_TRAP_WAIT_MS": "trap_wait_ms", "PM_LS_SPARSE": "ls_sparse", "PM_LS_SPARSE_T": "ls_sparse_T",
-        "PM_LS_CWALK": "ls_cwalk", "PM_LS_SPARSE_GMEM": "ls_sparse_gmem", "PM_AUCTION_GS": "auction_gs",
+        "PM_LS_CWALK": "ls_cwalk", "PM_LS_CWALK_C": "ls_cwalk_c", "PM_LS_SPARSE_GMEM": "ls_sparse_gmem", "PM_AUCTION_GS": "auction_gs",
         "PM_AUCTION_KEEP": "auction_keep", "PM_AUCTION_SMEM_PRICE": "auction_smem_price",
         "PM_AUCTION_THETA": "auction_theta", "PM_AUCTION_EPS_SHIFT": "auction_eps_shift",
         "PM_AUCTION_MAX_ROUNDS": "auction_max_rounds", "PM_AUCTION_CTAS_PER_SM": "auction_ctas_per_sm"}
