@@ -297,7 +297,8 @@ int64_t pm_launch_count(void);
  *   name  : one of "trap_variant" (chunk geometry 0..5), "trap_W" (owned
  *           pairs per chunk), "trap_cluster" (0 grid, 1 cluster), "trap_nbsync",
  *           "trap_cpc", "trap_ep" (sigma-permuted staging: 0 off, 1 auto,
- *           2 always), "trap_vec", "trap_spec", "trap_prefetch", "trap_prof",
+ *           2 always), "trap_vec", "trap_spec" (speculative class steps: 0 off, 1 quiet rounds,
+ *           2 always), "trap_coal" (warp-cooperative staging), "trap_prof",
  *           "trap_wait_ms" (bound of the multi-GPU waits, default 20000),
  *           "ls_sparse" (0: no sparse rounds), "ls_sparse_T" (hand-over swap
  *           count), "ls_cwalk" (0 one-CTA walk, 1 cluster walk),

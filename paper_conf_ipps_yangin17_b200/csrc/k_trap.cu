@@ -73,9 +73,6 @@ struct TrapParams {
   int64_t ldp;
   int32_t prof;                // trap_prof: CTA 0 thread 0 phase timers -> per_round[192..196]
   int32_t spec;                // speculative class steps (trap_spec, default 1)
-  int32_t prefetch;            // L2 prefetch of the next phases' E runs (trap_prefetch, default 1)
-  int32_t exp;
-  int32_t fstride;             // chunk flag spacing (uint32 units)
   int32_t coal;                // warp-cooperative (coalesced) staging of the Ep runs
   unsigned int* bar;           // grid barrier counter (zeroed before launch)
   unsigned long long* rsw;     // [3] swaps per round, rotating (grid mode)
@@ -156,9 +153,6 @@ __device__ __forceinline__ void stage_span(int32_t* dst, const int32_t* row, int
       cp_async4(dst + q, row + y);
     }
   }
-}
-__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
@@ -244,8 +238,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
                                           const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
                                           int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
                                           bool vec, unsigned long long* tprof,
-                                          const int32_t* __restrict__ Ep, int64_t ldp, bool spec, bool pf, int exp = 0,
-                                          bool coal = false) {
+                                          const int32_t* __restrict__ Ep, int64_t ldp, bool spec, bool coal) {
   using SM = TrapSmem<PPL, T, EP>;
   static_assert(T <= 64, "one mask bit per class of a phase");
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
@@ -292,31 +285,15 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       const int32_t* prow = Ep + (int64_t)g * ldp;
       offA[i] = (int32_t)((int64_t)g * ldp + (sp & ~3));
       offB[i] = (int32_t)((int64_t)g * ldp + (ss & ~3));
-      if (!(exp & 2) && !coal) {
-      if (!(exp & 16)) for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + q, prow + (sp & ~3) + q);
-      if (!(exp & 8)) for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + SM::SP + q, prow + (ss & ~3) + q);
-      }
-      if (pf && !fx) {
-        // the tile's partner runs of the next two phases continue this one
-        // (sigma(p0 + 2T) = sigma(p0) + T): pull them into L2 now, so the
-        // next stagings find them there if the tile stays (a hint only)
-        int32_t sn = sp + T;
-        sn = sn >= m ? sn - m : sn;
-        const int64_t nb = min((int64_t)(2 * SM::SPP * 4), 4 * (ldp - (sn & ~3))) & ~15ll;   // inside the row
-        if (nb >= 16) prefetch_l2(prow + (sn & ~3), (uint32_t)nb);
+      if (!coal) {
+        for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + q, prow + (sp & ~3) + q);
+        for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + SM::SP + q, prow + (ss & ~3) + q);
       }
     } else {
       s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
                    : make_int4(j | (2 << 16), d, j * RS + (p0 & 3), j * RS + SM::SP + (s0 & 3) + 2);
       stage_span(dst, row, p0 & ~3, SM::SP, m, vec);
       stage_span(dst + SM::SP, row, s0 & ~3, SM::SP, m, vec);
-      if (pf && !fx) {   // columns p0 + 2T .. p0 + 4T + 4 of the plain row (stride-2 runs)
-        int32_t cn = p0 + 2 * T;
-        cn = cn >= m ? cn - m : cn;
-        const int32_t c16 = cn & ~3;
-        const int32_t nb = min(4 * (2 * T + 8), 4 * (m - c16)) & ~15;
-        if (vec && nb >= 16) prefetch_l2(row + c16, (uint32_t)nb);
-      }
     }
     if (els[i] >= 0) dst[SM::CL] = els[i];          // carried by the published state (grid mode)
     else cp_async4(dst + SM::CL, row + (S - 1));
@@ -326,7 +303,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     // that paced the whole chunk chain: config 4 TRAP round 5.5 -> 5.0 ms.)
     if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, aligned || vec);
   }
-  if (EP && coal && !(exp & 2)) {
+  if (EP && coal) {
     // warp-cooperative copies of the runs of the warp's 32 slots: lane l of
     // copy `ins` moves 16-byte piece P = 32 ins + l of the warp's 64 runs, so
     // one warp instruction covers ~3.5 whole runs (contiguous pieces, ~18
@@ -352,7 +329,6 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
   if (spec && gt < 6) s_E[SM::MOFF + gt] = 0;
   cp_async_wait_all();
   group_sync(bar_id, GT);
-  if (exp & 4) return 0;
   unsigned long long t0 = tprof ? gtimer() : 0;
   // ---- Tp classes on the extended range: thread gt takes pair k = a + gt,
   // valid while t <= tmax (the trapezoid); its local slots are linear in t ----
@@ -557,11 +533,11 @@ k_ls_trap(const TrapParams p) {
             const int2* rr = rep + cur * S;
             mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { const int2 v = rr[x]; g = v.x; d = v.y; el = -1; },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.coal);
           } else {
             const int bi = p.nbsync ? (int)(qph % 3u) : cur;
             const int4* __restrict__ sc = bi == 0 ? p.sbuf[0] : (bi == 1 ? p.sbuf[1] : p.sbuf[2]);
-            if (p.nbsync && qph > 0 && !(p.exp & 1)) {
+            if (p.nbsync && qph > 0) {
               // the neighbour chunks' slots of phase qph - 1 (W >= 2T: every
               // reader of this buffer's previous generation is within two
               // chunks, and those finished it before our neighbours did theirs)
@@ -572,7 +548,7 @@ k_ls_trap(const TrapParams p) {
                   if (c2 < 0 || c2 >= p.nchunks) continue;
                   unsigned int v;
                   do {
-                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.flags + c2 * p.fstride) : "memory");
+                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p.flags + c2) : "memory");
                   } while (v < qph);
                 }
               }
@@ -582,7 +558,7 @@ k_ls_trap(const TrapParams p) {
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) {
                                          const int4 v = __ldcg(sc + x); g = v.x; d = v.y; el = v.z;
                                        },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.prefetch, p.exp, p.coal);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.coal);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
           // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
@@ -621,8 +597,8 @@ k_ls_trap(const TrapParams p) {
         if (prof) { const unsigned long long t = gtimer(); t_pub += t - tq; }
         group_sync(1 + grp, GT);
         if (!CLU && p.nbsync && have && gt == 0) {   // this chunk's slots of phase qph are out
-          if (!(p.exp & 32)) __threadfence();
-          asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.flags + ch * p.fstride), "r"(qph + 1u) : "memory");
+          __threadfence();
+          asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.flags + ch), "r"(qph + 1u) : "memory");
         }
       }
       // swaps of this phase -> the round counter
@@ -831,7 +807,7 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   // three generations of packed slot states (int4 [S] each)
   const size_t n = (size_t)S;
   ScopedScratch scr(st), ep(st);
-  const size_t head = (64 + sizeof(unsigned int) * (n / 2 + 16) * 32 + 15) / 16 * 16;
+  const size_t head = (64 + sizeof(unsigned int) * (n / 2 + 16) + 15) / 16 * 16;
   const size_t bytes = head + sizeof(int4) * 3 * n;
   PM_CUDA_TRY(pm::scratch_alloc(&scr.p, bytes, st));
   char* scratch = scr.as<char>();
@@ -850,11 +826,8 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
   hp.bar = bar; hp.rsw = rsw;
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.prof = knob("trap_prof", 0);
-  hp.exp = knob("trap_exp", 0);
-  hp.fstride = (hp.exp & 64) ? 32 : 1;
   hp.coal = knob("trap_coal", 1);
   hp.spec = knob("trap_spec", 1);
-  hp.prefetch = knob("trap_prefetch", 0);
   // sigma-permuted rows (the runs become contiguous: 5 instead of 9 16-byte
   // pieces per run at T = 16 from L2, dense sectors instead of stride-2 ones
   // from HBM)
@@ -932,7 +905,6 @@ struct TrapMultiParams {
   int32_t* handoff;               // the first rank's sparse-round flag (or NULL)
   int32_t sparse_T;
   int32_t spec;                   // speculative class steps
-  int32_t prefetch;               // L2 prefetch of the next phases' E runs
   int32_t coal;                   // coalesced staging of the Ep runs
   unsigned long long wait_ns;     // bound of every cross-rank wait
 };
@@ -1080,7 +1052,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
           const int32_t* __restrict__ dc = me.dbuf[bi];
           mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
                                      [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { g = __ldcg(rc + x); d = __ldcg(dc + x); el = -1; },
-                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp, spec, p.prefetch, 0, p.coal);
+                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp, spec, p.coal);
           // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
           int32_t own[3];
           int nown = 0;
@@ -1248,7 +1220,6 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   const bool coal_ok = (int64_t)S * ldp < (1ll << 31);
   hp.wait_ns = (unsigned long long)knob("trap_wait_ms", 20000) * 1000000ull;
   hp.spec = knob("trap_spec", 1);
-  hp.prefetch = knob("trap_prefetch", 0);
   hp.coal = coal_ok ? knob("trap_coal", 1) : 0;
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;

@@ -672,12 +672,15 @@ def test_multi_rank_trap_symmetric_memory_world1():
             tdist.destroy_process_group()
 
 
+@pytest.mark.parametrize("coal", [0, 1])
 @pytest.mark.parametrize("ep,mode", [("0", "1"), ("0", "0"), ("1", "0"), ("1", "1")])
-def test_trap_sigma_permuted_and_plain_row_staging(ep, mode):
+def test_trap_sigma_permuted_and_plain_row_staging(ep, mode, coal):
     # runs staged from the sigma-permuted copy of E (default while E is
-    # L2-resident) or from E's rows directly: identical results
+    # L2-resident), warp-cooperatively or one thread per tile, or from E's rows
+    # directly: identical results
     pm.tuning_set("trap_ep", int(ep))
     pm.tuning_set("trap_cluster", int(mode))
+    pm.tuning_set("trap_coal", coal)
     pm.tuning_set("ls_sparse", 0)
     _check_trap(oracle_E("smooth", 512, 16), mode == "1")
     _check_trap(oracle_E("ties", 128, 8), mode == "1")
