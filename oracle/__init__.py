@@ -22,6 +22,7 @@ serial_local_search(E)              Algorithm 1, P:118-129        (C)
 cost(E, r)                          Eq. (2), P:63                 (C)
 hungarian(E)                        Sec. III, Kuhn-Munkres P:102  (C, with dual certificate)
 render(I, M, r)                     the photomosaic image R, P:61/P:247 (C)
+histogram_match(I, T)               I's distribution adjusted to T's, reading R12 (C)
 brute_force(E)                      Eq. (3), all S! rearrangements (Python, S <= 8)
 
 Pins (tests/test_oracle_*.py) tie each of these to something other than
@@ -86,6 +87,8 @@ def _load():
     lib.or_hungarian.restype = ctypes.c_int32
     lib.or_render.argtypes = [_U8P, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _I32P, _U8P]
     lib.or_render.restype = None
+    lib.or_histogram_match.argtypes = [_U8P, _U8P, ctypes.c_int32, ctypes.c_int32, _U8P]
+    lib.or_histogram_match.restype = None
     lib.or_num_threads.argtypes = []
     lib.or_num_threads.restype = ctypes.c_int32
     lib.or_set_num_threads.argtypes = [ctypes.c_int32]
@@ -252,6 +255,19 @@ def render(I: np.ndarray, M: int, r: np.ndarray) -> np.ndarray:
     r = np.ascontiguousarray(r, dtype=np.int32)
     out = np.empty_like(a)
     _load().or_render(_p(a, _U8P), N, M, C, _p(r, _I32P), _p(out, _U8P))
+    return out if np.asarray(I).ndim == 3 else out[:, :, 0]
+
+
+# ---------------------------------------------------------------- P:84 -----
+def histogram_match(I: np.ndarray, T: np.ndarray) -> np.ndarray:
+    """I's intensity distribution adjusted to T's (Sec. II, P:84; reading
+    R12): per channel, level k -> the smallest level z with C_T(z) >= C_I(k)
+    (cumulative pixel counts).  Returns a new u8 image shaped like I."""
+    a, N, C = _img(I)
+    b, N2, C2 = _img(T)
+    assert (N, C) == (N2, C2)
+    out = np.empty_like(a)
+    _load().or_histogram_match(_p(a, _U8P), _p(b, _U8P), N, C, _p(out, _U8P))
     return out if np.asarray(I).ndim == 3 else out[:, :, 0]
 
 

@@ -311,3 +311,40 @@ void or_set_num_threads(int32_t t) {
   (void)t;
 #endif
 }
+
+/* ------------------------------------------------------------------------ */
+/* Histogram matching of the input image to the target (Sec. II: "the
+ * distribution of an input image is changed to that of a target image using
+ * the histogram equalization [10]").  Reading R12: histogram
+ * specification in its exact integer form, per channel c, L = 256 levels:
+ *   h_I[k], h_T[k]  = pixel counts of level k in channel c of I and T;
+ *   C_I[k], C_T[k]  = cumulative counts sum_{j <= k} h[j];
+ *   map[k]          = the smallest level z with C_T[z] >= C_I[k]
+ *                     (z = G^{-1}(T(k)) of [10] with the cumulative
+ *                     distributions compared as counts: both images have
+ *                     N*N pixels, so no division and no rounding);
+ *   out(y, x, c)    = map[I(y, x, c)].
+ * I, T, out: u8 [N][N][C] HWC; out may alias I.                            */
+void or_histogram_match(const uint8_t* I, const uint8_t* T, int32_t N, int32_t C, uint8_t* out) {
+  int64_t n = (int64_t)N * N;
+  for (int32_t c = 0; c < C; ++c) {
+    int64_t hI[256], hT[256], cI[256], cT[256];
+    uint8_t map[256];
+    for (int k = 0; k < 256; ++k) { hI[k] = 0; hT[k] = 0; }
+    for (int64_t p = 0; p < n; ++p) {
+      hI[I[p * C + c]] += 1;
+      hT[T[p * C + c]] += 1;
+    }
+    int64_t sI = 0, sT = 0;
+    for (int k = 0; k < 256; ++k) {
+      sI += hI[k]; cI[k] = sI;
+      sT += hT[k]; cT[k] = sT;
+    }
+    for (int k = 0; k < 256; ++k) {
+      int z = 0;
+      while (z < 255 && cT[z] < cI[k]) ++z;
+      map[k] = (uint8_t)z;
+    }
+    for (int64_t p = 0; p < n; ++p) out[p * C + c] = map[I[p * C + c]];
+  }
+}
