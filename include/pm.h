@@ -256,6 +256,21 @@ pm_status_t pm_photomosaic_host(const uint8_t* h_input, const uint8_t* h_target,
 pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, const int32_t* d_perm,
                       uint8_t* d_out, pm_stream_t stream);
 
+/* Adjusting the input image's intensity distribution to the target's before
+ * Step 1 (Sec. II: "the distribution of an input image is changed to
+ * that of a target image using the histogram equalization [10]"; reading
+ * R12): for every channel c separately, with C_I(k) and C_T(k) the numbers
+ * of pixels of level <= k in channel c of d_input and d_target,
+ *   d_out(y, x, c) = min{ z : C_T(z) >= C_I(d_input(y, x, c)) }
+ * (histogram specification on cumulative counts -- integers, no rounding).
+ *   d_input, d_target : u8 [N][N][C] HWC (the same N and C); C <= 4.
+ *   d_out : u8 [N][N][C]; may be d_input (in place), not d_target.
+ * Not part of pm_photomosaic*: the hot path takes its images as given
+ * (reading R12); call this first to reproduce the paper's preprocessing.
+ * Async on stream. */
+pm_status_t pm_histogram_match(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t C,
+                               uint8_t* d_out, pm_stream_t stream);
+
 /* The paper's optimization algorithm (Sec. III): the best
  * rearrangement R* (Eq. 3), i.e. a minimum-weight perfect matching of
  * the complete bipartite graph input tiles x target slots with

@@ -467,6 +467,14 @@ pm_status_t pm_render(const uint8_t* d_input, int32_t N, int32_t M, int32_t C, c
   return PM_OK;
 }
 
+pm_status_t pm_histogram_match(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t C,
+                               uint8_t* d_out, pm_stream_t stream) {
+  if (!d_input || !d_target || !d_out || N < 1 || C < 1) return PM_ERR_INVALID;
+  if (C > hist_max_channels()) return PM_ERR_UNSUPPORTED;
+  if (d_out == d_target && d_target != d_input) return PM_ERR_INVALID;   // the target is read after the input's map
+  return run_histogram_match(d_input, d_target, N, C, d_out, (cudaStream_t)stream);
+}
+
 pm_status_t pm_optimal_assignment(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm, int64_t* d_price,
                                   int32_t* h_rounds, int64_t* h_cost, pm_stream_t stream) {
   if (!d_E || !d_perm || S < 1 || ld_E < S) return PM_ERR_INVALID;

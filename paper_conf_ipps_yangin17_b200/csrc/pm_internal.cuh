@@ -207,6 +207,11 @@ pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* c
                             void* const* ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
                             LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
 
+// Histogram matching of I to T (k_hist.cu, reading R12).
+int32_t hist_max_channels();
+pm_status_t run_histogram_match(const uint8_t* I, const uint8_t* T, int32_t N, int32_t C, uint8_t* out,
+                                cudaStream_t st);
+
 // Exact min-weight perfect matching by eps-scaling auction (k_assign.cu).
 // h_stats (nullable): {bidding rounds, phases}.  Synchronises st.
 pm_status_t run_assignment(const int32_t* E, int64_t ld, int32_t S, int32_t* perm, int64_t* price_out,

@@ -48,6 +48,7 @@ _SIGS = [
     ("pm_photomosaic_host", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _I32, _P, _P, _P, _P, _P]),
     ("pm_render", ctypes.c_int, [_P, _I32, _I32, _I32, _P, _P, _P]),
     ("pm_optimal_assignment", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P, _P, _P]),
+    ("pm_histogram_match", ctypes.c_int, [_P, _P, _I32, _I32, _P, _P]),
     ("pm_launch_count", _I64, []),
     ("pm_trap_workspace_bytes", ctypes.c_size_t, [_I32]),
     ("pm_trap_workspace_reset", ctypes.c_int, [_P, _I32, _P]),
@@ -333,6 +334,26 @@ def render(I, M: int, perm, out=None, stream=None):
     if out is None:
         out = torch.empty_like(img)
     _check(lib().pm_render(img.data_ptr(), N, M, C, perm.data_ptr(), out.data_ptr(), _stream(stream)), "pm_render")
+    return out if I.dim() == 3 else out[:, :, 0]
+
+
+# ------------------------------------------------ histogram ---------
+def histogram_match(I, T, out=None, stream=None):
+    """pm_histogram_match: I's intensity distribution adjusted to T's (Sec. II,
+    P:84; reading R12).  Returns the adjusted image (out, or a new tensor;
+    out may be I for in-place)."""
+    torch = _torch()
+    img = _dev_u8_image(I)
+    tgt = _dev_u8_image(T)
+    if tgt.shape != img.shape:
+        raise ValueError("input and target must have the same shape (P:57)")
+    N, C = img.shape[0], img.shape[2]
+    if out is None:
+        out = torch.empty_like(img)
+    elif out.dim() == 2:
+        out = out.unsqueeze(-1)
+    _check(lib().pm_histogram_match(img.data_ptr(), tgt.data_ptr(), N, C, out.data_ptr(), _stream(stream)),
+           "pm_histogram_match")
     return out if I.dim() == 3 else out[:, :, 0]
 
 

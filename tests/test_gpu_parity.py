@@ -418,9 +418,12 @@ def test_error_matrix_simulated_8_shards_config4():
 
 
 # ------------------------------------------- NEXT-1: the paper's grayscale grid
-@pytest.mark.parametrize("N,g", [(512, 16), (512, 32), (1024, 16), (1024, 32), (2048, 16)])
+@pytest.mark.parametrize("N,g", [(512, 16), (512, 32), (512, 64), (1024, 16), (1024, 32), (1024, 64),
+                                 (2048, 16), (2048, 32), (2048, 64)])
 def test_paper_grid_grayscale_parity(N, g):
-    # Tables II-IV shapes, C = 1: tile sides 8..128 px, P up to 16384 bytes
+    # all nine Tables II-IV shapes, C = 1: grids 16^2 / 32^2 / 64^2
+    # (S = 256 / 1024 / 4096), tile sides 8..128 px, P up to 16384 bytes --
+    # E, r, rounds, swaps and cost against the oracle
     M = N // g
     I, T = pair("smooth", N, M, 1)
     Eg = pm.error_matrix(dev(I), dev(T), M)
@@ -429,18 +432,8 @@ def test_paper_grid_grayscale_parity(N, g):
     ref = oracle.local_search(E)
     perm, rounds, swaps, per, st = pm.local_search(Eg)
     assert (perm.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    assert (per == ref[3]).all()
     assert pm.cost(Eg, perm) == oracle.cost(E, ref[0])
-
-
-@pytest.mark.parametrize("N,g", [(512, 64), (2048, 64)])
-def test_paper_grid_grayscale_S4096_sampled(N, g):
-    # S = 64^2 = 4096 (the paper's largest grid): E sampled against the oracle,
-    # the search against the oracle replay run on the oracle's own E
-    M = N // g
-    I, T = pair("smooth", N, M, 1)
-    Eg = pm.error_matrix(dev(I), dev(T), M)
-    rng = np.random.default_rng(N)
-    _sampled_E_check(I, T, M, Eg, 0, rng, 400)
 
 
 # ------------------------------------------------- NEXT-3: render R --
