@@ -637,10 +637,11 @@ int32_t ls_sparse_threshold(int32_t S, int32_t dense_method) {
   // 2489-swap round, 27 vs 33 ms; S = 16384: after the 4715-swap round,
   // 240 vs 375 ms at S^2/1024).
   // TRAP dense rounds: hand over after the first round with <= 256 swaps up to
-  // S = 16384, <= S/8 beyond (measured: config 4 whole search
-  // 37.2 ms at 256 vs 39.7 at 1024, 39.0 at 128, 42.0 at 64; configs 2/3
-  // best at 256 too)
-  if (dense_method == PM_LS_TRAP) return S <= 16384 ? 256 : S / 8;
+  // S = 16384, <= 32 beyond (measured: config 4 whole search 28.3
+  // ms at 256 vs 30.1 at 128, 32.7 at 64; configs 2/3 best at 256 too;
+  // config 5 584 ms at 32 vs 633-1351 at S/8 = 8192 -- its walk keeps the
+  // replicas in global memory and every gather goes to HBM)
+  if (dense_method == PM_LS_TRAP) return S <= 16384 ? 256 : 32;
   if (S > 2048) return (int32_t)((int64_t)S * 3 / 4);
   const int64_t t2 = (int64_t)S * S / 1024;
   return (int32_t)(t2 < 1 ? 1 : (t2 > INT32_MAX ? INT32_MAX : t2));

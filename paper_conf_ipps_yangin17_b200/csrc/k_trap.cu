@@ -48,6 +48,7 @@
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdio>
 #include <cstdlib>
 
@@ -252,7 +253,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
   // flight together) ----
   constexpr int NJ = (SM::L + GT - 1) / GT;   // slots per thread (2)
   int32_t xs[NJ], gs[NJ], ds[NJ], els[NJ];   // els: E[g][S-1] when the state carries it, else -1
-  int32_t offA[NJ], offB[NJ];                 // coalesced staging: element offsets of the two runs in Ep
+  int32_t colA[NJ], colB[NJ];                 // coalesced staging: start columns of the two runs in Ep
 #pragma unroll
   for (int i = 0; i < NJ; ++i) {
     const int32_t j = gt + i * GT;
@@ -283,8 +284,8 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
                    : make_int4(j | (1 << 16), d, j * RS + (sp & 3), j * RS + SM::SP + (ss & 3) + 1);
       const int32_t* prow = Ep + (int64_t)g * ldp;
-      offA[i] = (int32_t)((int64_t)g * ldp + (sp & ~3));
-      offB[i] = (int32_t)((int64_t)g * ldp + (ss & ~3));
+      colA[i] = sp & ~3;
+      colB[i] = ss & ~3;
       if (!coal) {
         for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + q, prow + (sp & ~3) + q);
         for (int32_t q = 0; q < SM::SPP; q += 4) cp_async16(dst + SM::SP + q, prow + (ss & ~3) + q);
@@ -319,10 +320,12 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
         const int r = P / NP;                 // run of the warp: 2 per slot
         const int q = P - r * NP;
         const int sl = r >> 1;
-        const int32_t oA = __shfl_sync(0xffffffffu, offA[i], sl);
-        const int32_t oB = __shfl_sync(0xffffffffu, offB[i], sl);
+        const int32_t gr = __shfl_sync(0xffffffffu, gs[i], sl);
+        const int32_t cA = __shfl_sync(0xffffffffu, colA[i], sl);
+        const int32_t cB = __shfl_sync(0xffffffffu, colB[i], sl);
         const int32_t js = wbase + sl + i * GT;
-        if (js < Lc) cp_async16(s_E + js * RS + ((r & 1) ? SM::SP : 0) + 4 * q, Ep + ((r & 1) ? oB : oA) + 4 * q);
+        if (js < Lc)
+          cp_async16(s_E + js * RS + ((r & 1) ? SM::SP : 0) + 4 * q, Ep + (int64_t)gr * ldp + ((r & 1) ? cB : cA) + 4 * q);
       }
     }
   }
@@ -773,19 +776,40 @@ static pm_status_t launch_trap_ep(TrapParams& hp, cudaStream_t st) {
   return PM_OK;
 }
 
-// sigma-permuted copy of E: up to E = 2 GiB (trap_ep 1, measured: config 2
-// 1.25 -> 1.18 ms, config 4 67.4 -> 62.3 ms; config 5 1.09 -> 1.25 s --
-// building the 16 GiB copy costs more than it saves), always (2), never (0).
-// The runs become contiguous: dense sectors instead of stride-2 ones.
+// sigma-permuted copy of E (trap_ep: 1 auto, 2 always, 0 never).  Auto
+// builds it whenever it takes at most 1/8 of the device's memory (22 GiB on
+// a B200, E itself being as large; the total is queried once per device --
+// cudaMemGetInfo per call costs ~0.6 ms and synchronises): since the staging
+// became warp-cooperative and the 192 x 48 geometry needs its compact rows,
+// it pays at every size (config 5, measured: whole search 970 ms from E's
+// rows with 64 x 16 chunks vs 584 ms with the 16 GiB copy and 192 x 48; in
+// round 1, before both, it lost there: 1.09 vs 1.25 s).
+static size_t device_total_mem() {
+  static std::atomic<size_t> totals[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 0;
+  size_t t = totals[dev].load();
+  if (t == 0) {
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, dev) != cudaSuccess) return 0;
+    t = prop.totalGlobalMem;
+    totals[dev].store(t);
+  }
+  return t;
+}
+
 pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
-                                 int64_t* ldp) {
+                          int64_t* ldp) {
   *Ep = nullptr;
   *ldp = 0;
   const int32_t ep_mode = knob("trap_ep", 1);
-  if (ep_mode == 0 || (ep_mode == 1 && (int64_t)S * ldE * 4 > (2ll << 30))) return PM_OK;
+  if (ep_mode == 0) return PM_OK;
   const int32_t m = S - 1, ext = 48;
-  *ldp = ((int64_t)m + ext + 31) / 32 * 32;
-  PM_CUDA_TRY(pm::scratch_alloc(Ep, sizeof(int32_t) * (size_t)S * (size_t)*ldp, st));
+  const int64_t l = ((int64_t)m + ext + 31) / 32 * 32;
+  const size_t bytes = sizeof(int32_t) * (size_t)S * (size_t)l;
+  if (ep_mode == 1 && bytes > device_total_mem() / 8) return PM_OK;
+  *ldp = l;
+  PM_CUDA_TRY(pm::scratch_alloc(Ep, bytes, st));
   PM_CUDA_TRY(launch_permute_cols(E, ldE, *Ep, *ldp, S, m, ext, st));
   return PM_OK;
 }
@@ -843,7 +867,6 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
     if (se != PM_OK) return se;
     hp.Ep = Ep; hp.ldp = ldp;
   }
-  if (hp.Ep && (int64_t)S * hp.ldp >= (1ll << 31)) hp.coal = 0;   // int32 element offsets
   // 16-byte span copies pay while E is L2-resident (config 2/3 staging 2.55 ->
   // 1.80 / 3.2 -> 2.1 us per phase); from HBM the 4-byte entry copies of the
   // used runs win (config 4: 5.0 vs 10.8 us)
@@ -1217,10 +1240,9 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   hp.out = dev_out; hp.per_round = dev_per_round;
   hp.handoff = handoff; hp.sparse_T = sparse_T;
   hp.ldp = ldp;
-  const bool coal_ok = (int64_t)S * ldp < (1ll << 31);
   hp.wait_ns = (unsigned long long)knob("trap_wait_ms", 20000) * 1000000ull;
   hp.spec = knob("trap_spec", 1);
-  hp.coal = coal_ok ? knob("trap_coal", 1) : 0;
+  hp.coal = knob("trap_coal", 1);
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
   int max_cpc = (int)((size_t)optin / SM::bytes);
@@ -1246,11 +1268,11 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
 
 static int32_t trap_multi_variant(int32_t S, int64_t ldE) {
   int32_t v = knob("trap_variant", -1);
-  if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20) && S <= 16384) ? 5 : 0;
+  if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20)) ? 5 : 0;
   return v;
 }
-// Chunk geometry as the single-GPU grid mode: 64 x 16 while E is
-// L2-resident or S > 16384, else 128 x 32 (PM_TRAP_V = 0 / 5 force one).
+// Chunk geometry: 64 x 16 while E is L2-resident (small S: enough chunks for
+// every rank), else 128 x 32 (trap_variant 0 / 5 force one).
 pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
                            int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                            cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0, int64_t ldp = 0) {

@@ -39,5 +39,5 @@ for cfg in cfgs:
         same = "" if ref is None else ("same" if res == ref else "DIFFERENT")
         ref = ref or res
         ts.sort()
-        print(f"cfg{cfg} S={S} {m:7s} {ts[len(ts)//2]:9.3f} ms  rounds={rounds} swaps={swaps} "
+        print(f"cfg{cfg} S={S} {m:7s} {ts[len(ts)//2]:9.3f} ms [min {ts[0]:.3f} max {ts[-1]:.3f}] rounds={rounds} swaps={swaps} "
               f"ns/class-step={ts[len(ts)//2]*1e6/(rounds*(S-1)):.0f} per_round={per.tolist()} {same}", flush=True)
