@@ -1266,18 +1266,30 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   return PM_OK;
 }
 
+static bool ep_expected(int32_t S) {   // trap_build_ep's rule, before anything is allocated
+  const int32_t mode = knob("trap_ep", 1);
+  if (mode == 0) return false;
+  const int64_t l = ((int64_t)S - 1 + 48 + 31) / 32 * 32;
+  return mode == 2 || sizeof(int32_t) * (size_t)S * (size_t)l <= device_total_mem() / 8;
+}
 static int32_t trap_multi_variant(int32_t S, int64_t ldE) {
   int32_t v = knob("trap_variant", -1);
-  if (v != 0 && v != 5) v = ((int64_t)S * ldE * 4 > (96ll << 20)) ? 5 : 0;
+  if (v != 0 && v != 5 && v != 6)
+    v = ((int64_t)S * ldE * 4 > (96ll << 20)) ? (ep_expected(S) ? 6 : 5) : 0;
   return v;
 }
-// Chunk geometry: 64 x 16 while E is L2-resident (small S: enough chunks for
-// every rank), else 128 x 32 (trap_variant 0 / 5 force one).
+// Chunk geometry as the single-GPU path: 64 x 16 while E is L2-resident
+// (small S: enough chunks for every rank), else 192 x 48 with the
+// sigma-permuted copy, 128 x 32 without (trap_variant 0 / 5 / 6 force one).
 pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE, int32_t S,
                            int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
                            cudaStream_t st, int32_t* handoff = nullptr, int32_t sparse_T = 0, int64_t ldp = 0) {
   const bool ep = ranks[rank0].Ep != nullptr;
-  if (trap_multi_variant(S, ldE) == 5)
+  const int32_t v = trap_multi_variant(S, ldE);
+  if (v == 6 && ep)
+    return launch_trap_multi<6, 48, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                          max_log, st, handoff, sparse_T, ldp);
+  if (v == 5 || v == 6)
     return ep ? launch_trap_multi<4, 32, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
                                                max_log, st, handoff, sparse_T, ldp)
               : launch_trap_multi<4, 32, false>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
@@ -1294,7 +1306,8 @@ pm_status_t run_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_
 pm_status_t trap_multi_supported(int32_t S, int64_t ldE, int32_t world) {
   if (world < 1 || world > kMaxRanks) return PM_ERR_INVALID;
   if (S < ls_trap_min_S() || (S & 1)) return PM_ERR_UNSUPPORTED;
-  const int32_t W = trap_multi_variant(S, ldE) == 5 ? 64 : 32;   // X - 2T of the geometry
+  const int32_t v = trap_multi_variant(S, ldE);
+  const int32_t W = v == 6 ? 96 : (v == 5 ? 64 : 32);   // X - 2T of the geometry
   if ((Classes(S).npairs + W - 1) / W < world) return PM_ERR_UNSUPPORTED;
   return PM_OK;
 }
@@ -1321,22 +1334,22 @@ pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_
     PM_CUDA_TRY(cudaMemcpyAsync(pr, perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
     trap_ws_layout(ws, S, pr, E, ranks[r]);
   }
-  // quiet rounds: every rank would continue alone with the same sparse
-  // rounds; here rank world-1 (the farthest from the launch's first) does
-  const int32_t sparse_T = ls_sparse_threshold(S, PM_LS_TRAP);
-  SparseRun sr;
-  if (sparse_T > 0) {
-    const pm_status_t s0 = sparse_prepare(E, ldE, S, ranks[world - 1].perm, max_rounds, dev_out, dev_per_round,
-                                          max_log, st, &sr);
-    if (s0 != PM_OK) return s0;
-    sps.p = sr.scratch;   // freed here on an error path; sparse_launch frees it otherwise
-  }
   int64_t ldp = 0;
   {
     int32_t* Ep = nullptr;
     const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
     ep.p = Ep;
     if (se != PM_OK) return se;
+  }
+  // quiet rounds: every rank would continue alone with the same sparse
+  // rounds; here rank world-1 (the farthest from the launch's first) does
+  const int32_t sparse_T = ls_sparse_threshold(S, PM_LS_TRAP);
+  SparseRun sr;
+  if (sparse_T > 0) {
+    const pm_status_t s0 = sparse_prepare(E, ldE, S, ranks[world - 1].perm, max_rounds, dev_out, dev_per_round,
+                                          max_log, st, &sr, 0, ep.as<int32_t>(), ldp);
+    if (s0 != PM_OK) return s0;
+    sps.p = sr.scratch;   // freed here on an error path; sparse_launch frees it otherwise
   }
   for (int r = 0; r < world; ++r) ranks[r].Ep = ep.as<int32_t>();
   pm_status_t s = run_trap_multi(ranks, world, 0, world, ldE, S, max_rounds, dev_out, dev_per_round, max_log, st,
@@ -1372,19 +1385,19 @@ pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* c
   // of r and E -- every rank reaches the same result, no exchange)
   const int32_t sparse_T = ls_sparse_threshold(S, PM_LS_TRAP);
   ScopedScratch sps(st), ep(st);
-  SparseRun sr;
-  if (sparse_T > 0) {
-    const pm_status_t s0 = sparse_prepare(E, ldE, S, perm_peers[rank], max_rounds, dev_out, dev_per_round, max_log,
-                                          st, &sr);
-    if (s0 != PM_OK) return s0;
-    sps.p = sr.scratch;
-  }
   int64_t ldp = 0;
   {
     int32_t* Ep = nullptr;
     const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
     ep.p = Ep;
     if (se != PM_OK) return se;
+  }
+  SparseRun sr;
+  if (sparse_T > 0) {
+    const pm_status_t s0 = sparse_prepare(E, ldE, S, perm_peers[rank], max_rounds, dev_out, dev_per_round, max_log,
+                                          st, &sr, 0, ep.as<int32_t>(), ldp);
+    if (s0 != PM_OK) return s0;
+    sps.p = sr.scratch;
   }
   ranks[rank].Ep = ep.as<int32_t>();   // only this rank's entry is read by this launch
   const pm_status_t s = run_trap_multi(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, dev_per_round, max_log,

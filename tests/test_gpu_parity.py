@@ -623,7 +623,7 @@ def test_multi_rank_trap_emulated(N, M, fam, world):
     assert (rounds, swaps) == (ref[1], ref[2])
 
 
-@pytest.mark.parametrize("variant", ["0", "5"])
+@pytest.mark.parametrize("variant", ["0", "5", "6"])
 def test_multi_rank_trap_geometries(variant):
     pm.tuning_set("trap_variant", int(variant))
     E_np = oracle_E("smooth", 1024, 16)
