@@ -254,10 +254,9 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
   }
 }
 
-// Host-side tiling choice: 128 x 128 tiles with split-K over the divisors of
-// nkb, or 128 x 64 tiles (two CTAs per SM, half the work per tile) without
-// split-K.  Cost = waves * per-CTA work, with a small bias against split-K
-// (its memset and atomics).
+// Host-side tiling choice: 128 x 128 or 128 x 64 tiles (two CTAs per SM,
+// half the work per tile), each with split-K over the divisors of nkb.
+// Cost = waves * per-CTA work, biased by measured factors.
 struct SadPlan { int bn, split; };
 static SadPlan choose_plan(int64_t nrows, int64_t S, int nkb, int sms) {
   SadPlan best{128, 1};
@@ -267,13 +266,25 @@ static SadPlan choose_plan(int64_t nrows, int64_t S, int nkb, int sms) {
     if (nkb % s) continue;
     if (s > 1 && nkb / s < 2) break;
     const int64_t ctas = gy * ((S + 127) / 128) * s;
-    const double cost = (double)((ctas + sms - 1) / sms) * (nkb / s) * (s > 1 ? 1.10 : 1.0);
+    const double cost = (double)((ctas + sms - 1) / sms) * (nkb / s) * (s > 1 ? 1.35 : 1.0);
     if (cost < best_cost - 1e-9) { best_cost = cost; best = {128, s}; }
   }
-  {
-    const int64_t ctas = gy * ((S + 63) / 64);
-    const double cost = (double)((ctas + sms - 1) / sms) * nkb * 0.5;   // half-size tiles (two per SM hide latency)
-    if (cost < best_cost - 1e-9) { best_cost = cost; best = {64, 1}; }
+  // half-size tiles, two CTAs per SM.  Factors measured (round 2, configs
+  // 2-4, tools/e_bench.py): 128 x 64 tiles are ~3 % faster than 128 x 128 at
+  // any size (0.48 per half-size tile), and split-K never paid (its memset
+  // and atomics: x1.35)
+  for (int s = 1; s <= nkb; ++s) {
+    if (nkb % s) continue;
+    if (s > 1 && nkb / s < 2) break;
+    const int64_t ctas = gy * ((S + 63) / 64) * s;
+    const double cost = (double)((ctas + sms - 1) / sms) * (nkb / s) * 0.48 * (s > 1 ? 1.35 : 1.0);
+    if (cost < best_cost - 1e-9) { best_cost = cost; best = {64, s}; }
+  }
+  // tuning: sad_plan = 1000 * bn + split forces a plan (tests / tools)
+  const int32_t forced = knob("sad_plan", 0);
+  if (forced > 0) {
+    const int bn = forced / 1000 == 64 ? 64 : 128, sp = forced % 1000;
+    if (sp >= 1 && nkb % sp == 0) best = {bn, sp};
   }
   return best;
 }
@@ -300,6 +311,8 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
     if ((e = sad_set_attr<true, true, 128>()) != cudaSuccess) return e;
     if ((e = sad_set_attr<false, false, 64>()) != cudaSuccess) return e;
     if ((e = sad_set_attr<false, true, 64>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<true, false, 64>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr<true, true, 64>()) != cudaSuccess) return e;
     attr_done.fetch_or(1ull << dev);
   }
   const int kw = image ? P / 4 : (int)(geo.ldt / 4);
@@ -307,21 +320,28 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
   const int64_t gy = (nrows + BM - 1) / BM;
   if (gy > 65535) return cudaErrorInvalidValue;
   const SadPlan plan = choose_plan(nrows, S, nkb, sms);
-  if (plan.bn == 64) {
-    dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, 1);
-    if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
-    else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
-    note_launch();
-    return cudaGetLastError();
-  }
   const int split = plan.split;
-  dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
   if (split > 1) {
     // split-K accumulates with red.add: zero the [nrows][S] window of E first
     cudaError_t e = (ldE == S)
         ? cudaMemsetAsync(E, 0, sizeof(int32_t) * (size_t)nrows * S, st)
         : cudaMemset2DAsync(E, sizeof(int32_t) * ldE, 0, sizeof(int32_t) * S, nrows, st);
     if (e != cudaSuccess) return e;
+  }
+  if (plan.bn == 64) {
+    dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, (unsigned)split);
+    if (split > 1) {
+      if (image) k_sad<true, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE);
+      else k_sad<true, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE);
+    } else {
+      if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
+      else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
+    }
+    note_launch();
+    return cudaGetLastError();
+  }
+  dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
+  if (split > 1) {
     if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE);
     else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE);
   } else {

@@ -52,7 +52,7 @@ static std::map<std::string, int32_t> g_tune;
 
 static const char* const kTuningNames[] = {
     "trap_variant", "trap_W", "trap_cluster", "trap_nbsync", "trap_cpc", "trap_prof", "trap_ep", "trap_vec",
-    "trap_spec",    "trap_wait_ms", "trap_coal",
+    "trap_spec",    "trap_wait_ms", "trap_coal", "sad_plan",
     "ls_sparse",    "ls_sparse_T", "ls_cwalk", "ls_sparse_gmem", "ls_cwalk_c",
     "auction_gs",   "auction_keep", "auction_smem_price", "auction_theta", "auction_eps_shift",
     "auction_max_rounds", "auction_ctas_per_sm"};

@@ -72,6 +72,15 @@ def test_error_matrix_parity(fam, N, M, C):
     assert (E == oracle_E(fam, N, M, C)).all()
 
 
+@pytest.mark.parametrize("plan", [64001, 64002, 64003, 64004, 128001, 128002, 128003])
+@pytest.mark.parametrize("N,M,C,fam", [(512, 16, 3, "noise"), (90, 10, 3, "smooth"), (256, 16, 1, "ties")])
+def test_error_matrix_every_tiling_plan(plan, N, M, C, fam):
+    # 128 x 128 and 128 x 64 tiles, with and without split-K (exact red.add)
+    pm.tuning_set("sad_plan", plan)
+    I, T = pair(fam, N, M, C)
+    assert (pm.error_matrix(dev(I), dev(T), M).cpu().numpy() == oracle_E(fam, N, M, C)).all()
+
+
 def test_error_matrix_config3_full():
     # n = 4096, no split-K path, 32 x 32 CTA tiles
     E = pm.error_matrix(*map(dev, pair("smooth", 1024, 16)), 16).cpu().numpy()

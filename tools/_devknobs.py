@@ -6,7 +6,7 @@ import os
 _MAP = {"PM_TRAP_V": "trap_variant", "PM_TRAP_W": "trap_W", "PM_TRAP_CLUSTER": "trap_cluster",
         "PM_TRAP_NBSYNC": "trap_nbsync", "PM_TRAP_CPC": "trap_cpc", "PM_TRAP_PROF": "trap_prof",
         "PM_TRAP_EP": "trap_ep", "PM_TRAP_VEC": "trap_vec", "PM_TRAP_SPEC": "trap_spec",
-        "PM_TRAP_COAL": "trap_coal",
+        "PM_TRAP_COAL": "trap_coal", "PM_SAD_PLAN": "sad_plan",
         "PM_TRAP_WAIT_MS": "trap_wait_ms", "PM_LS_SPARSE": "ls_sparse", "PM_LS_SPARSE_T": "ls_sparse_T",
         "PM_LS_CWALK": "ls_cwalk", "PM_LS_CWALK_C": "ls_cwalk_c", "PM_LS_SPARSE_GMEM": "ls_sparse_gmem", "PM_AUCTION_GS": "auction_gs",
         "PM_AUCTION_KEEP": "auction_keep", "PM_AUCTION_SMEM_PRICE": "auction_smem_price",
