@@ -1127,11 +1127,12 @@ k_ls_trap_mr(const TrapMultiParams p) {
         // round end: every CTA's count to every rank's total (system-scope
         // atomics: the adds of several GPUs meet in one counter), then the
         // rank barrier and the cross-rank barrier, then the rank barrier again
-        if (threadIdx.x == 0 && s_cta_sw) {
-          for (int o = 0; o < world; ++o)
-            atomicAdd_system(p.rk[o].rtot + rounds % 3, (unsigned long long)s_cta_sw);
+        if (threadIdx.x == 0) {   // (thread 0 alone reads and resets the CTA's count)
+          const int cta_sw = s_cta_sw;
+          if (cta_sw)
+            for (int o = 0; o < world; ++o) atomicAdd_system(p.rk[o].rtot + rounds % 3, (unsigned long long)cta_sw);
+          s_cta_sw = 0;
         }
-        if (threadIdx.x == 0) s_cta_sw = 0;
         bar_target += nloc;
         if (!grid_barrier_mr(p, r, me.bar, bar_target)) { ok = false; break; }
         if (leader) {
