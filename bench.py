@@ -71,6 +71,9 @@ def parse():
     ap.add_argument("--independent", action="store_true",
                     help="N > 1: N independent photomosaics (weak scaling) instead of one sharded one")
     ap.add_argument("--sharded", action="store_true", help="N = 1: force the sharded code path")
+    ap.add_argument("--e-layout", default="gathered", choices=["gathered", "rows"],
+                    help="one photomosaic over N ranks: E all-gathered onto every rank (default), or left "
+                         "row-sharded in symmetric memory and read over NVLink (pm_local_search_sharded_async)")
     return ap.parse_args()
 
 
@@ -365,7 +368,10 @@ def bench_single(args, rank, world, local_rank):
 def bench_sharded(args, rank, world, local_rank):
     """One photomosaic for the whole job: every rank computes its row shard of
     E (pm_error_matrix rows), NCCL all-gathers E, and Algorithm 2 runs across
-    the ranks (pm_local_search_multi_async).  value = S^2 / step time."""
+    the ranks (pm_local_search_multi_async).  value = S^2 / step time.
+    --e-layout rows: E is never gathered -- each rank's rows stay in its
+    symmetric-memory shard and pm_local_search_sharded_async /
+    pm_cost_sharded_async read every row from its owner over NVLink."""
     import torch
     import torch.distributed as dist
     import torch.distributed._symmetric_memory as symm_mem
@@ -389,15 +395,24 @@ def bench_sharded(args, rank, world, local_rank):
     b, e = pdist.shard_rows(S, world, rank)
     sizes = [pdist.shard_rows(S, world, g) for g in range(world)]
     rows_max = max(se - sb for sb, se in sizes)
-    parts = torch.zeros((world, rows_max, S), dtype=torch.int32, device=dev)
-    part = parts[rank]                                                   # in-place all-gather
-    contiguous = all(se - sb == rows_max for sb, se in sizes)
-    E_full = parts.view(world * rows_max, S) if contiguous else torch.empty((S, S), dtype=torch.int32, device=dev)
-    ws_bytes = (pm.trap_workspace_bytes(S) + 255) // 256 * 256
-    buf = symm_mem.empty(ws_bytes + 4 * S, dtype=torch.uint8, device=dev)
+    rows_layout = args.e_layout == "rows"
+    pb = (4 * S + 255) // 256 * 256
+    if rows_layout:
+        rb = [sb for sb, _ in sizes] + [S]
+        ws_bytes = (pm.trap_workspace_bytes_sharded(S, rows_max) + 255) // 256 * 256
+        buf = symm_mem.empty(ws_bytes + pb + 4 * rows_max * S, dtype=torch.uint8, device=dev)
+        part = buf[ws_bytes + pb:].view(torch.int32).view(rows_max, S)     # this rank's shard, peer-mapped
+    else:
+        parts = torch.zeros((world, rows_max, S), dtype=torch.int32, device=dev)
+        part = parts[rank]                                               # in-place all-gather
+        contiguous = all(se - sb == rows_max for sb, se in sizes)
+        E_full = parts.view(world * rows_max, S) if contiguous else torch.empty((S, S), dtype=torch.int32, device=dev)
+        ws_bytes = (pm.trap_workspace_bytes(S) + 255) // 256 * 256
+        buf = symm_mem.empty(ws_bytes + pb, dtype=torch.uint8, device=dev)
     hdl = symm_mem.rendezvous(buf, dist.group.WORLD.group_name)
     ptrs = [int(p) for p in hdl.buffer_ptrs]
-    my_perm = buf[ws_bytes:].view(torch.int32)
+    my_perm = buf[ws_bytes:ws_bytes + 4 * S].view(torch.int32)
+    e_ptrs = [p + ws_bytes + pb for p in ptrs]
     res = torch.zeros(3, dtype=torch.int64, device=dev)
     cost = torch.zeros(1, dtype=torch.int64, device=dev)
     token = torch.zeros(1, dtype=torch.int32, device=dev)
@@ -412,7 +427,7 @@ def bench_sharded(args, rank, world, local_rank):
         if evs: evs[0].record(stream)
         pm.error_matrix(dI, dT, M, rows=(b, e), out=part[: e - b])        # Step 1+2, this rank's rows
         if evs: evs[1].record(stream)
-        if world > 1:
+        if world > 1 and not rows_layout:
             dist.all_gather_into_tensor(parts.view(world * rows_max, S), part)
             if not contiguous:
                 for g, (sb, se) in enumerate(sizes):
@@ -420,10 +435,16 @@ def bench_sharded(args, rank, world, local_rank):
         if evs: evs[2].record(stream)
         pm.init_identity(my_perm)
         pm.trap_workspace_reset(buf, S)
-        dist.all_reduce(token)                                             # every workspace reset (device order)
-        pm.local_search_multi_async(E_full, [p + ws_bytes for p in ptrs], ptrs, rank, world, res)
+        dist.all_reduce(token)                             # every workspace reset, every shard written (device order)
+        if rows_layout:
+            pm.local_search_sharded_async(e_ptrs, rb, S, S, [p + ws_bytes for p in ptrs], ptrs, rank, world, res)
+        else:
+            pm.local_search_multi_async(E_full, [p + ws_bytes for p in ptrs], ptrs, rank, world, res)
         if evs: evs[3].record(stream)
-        pm.cost_async(E_full, my_perm, cost)
+        if rows_layout:
+            pm.cost_sharded_async(e_ptrs, rb, S, S, my_perm, cost)
+        else:
+            pm.cost_async(E_full, my_perm, cost)
         if evs: evs[4].record(stream)
         if host:                                                           # e2e: host r out
             hperm.copy_(my_perm, non_blocking=True)
@@ -469,16 +490,22 @@ def bench_sharded(args, rank, world, local_rank):
         "metric": METRIC, "value": S * S / (ms * 1e-3) / 1e9, "unit": UNIT, "n_gpus": world, "steps": K,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "u8->int32", "data": "synthetic",
-        "config": dict(workload_desc(args.config, args.family, [0]), method="trap (multi-rank)",
-                       parallelism=f"one photomosaic: E rows sharded over {world} ranks + NCCL all-gather; "
-                                   f"Alg. 2 across the ranks (NVLink peer stores of halo slots)",
+        "config": dict(workload_desc(args.config, args.family, [0]),
+                       method="trap (multi-rank, row-sharded E)" if rows_layout else "trap (multi-rank)",
+                       parallelism=(f"one photomosaic: E rows sharded over {world} ranks, never gathered; Alg. 2 "
+                                    f"across the ranks reading E rows from their owner (NVLink peer loads)"
+                                    if rows_layout else
+                                    f"one photomosaic: E rows sharded over {world} ranks + NCCL all-gather; "
+                                    f"Alg. 2 across the ranks (NVLink peer stores of halo slots)"),
                        l2="flushed between steps (512 MiB write outside the per-step CUDA events)"),
         "gpairs_per_s_error_matrix": S * S / (pdist.max_over_ranks(part_ms["error_matrix_shard"], device=dev)
                                               * 1e-3) / 1e9,
         "e2e": {"value": S * S / (e2e_ms * 1e-3) / 1e9, "unit": UNIT, "ms": e2e_ms,
                 "h2d_bytes_per_step": 2 * N * N * C, "d2h_bytes_per_step": 4 * S,
-                "api": "per rank: pinned host images -> pm_error_matrix rows -> all-gather -> "
-                       "pm_local_search_multi_async -> pm_cost_async -> pinned host r"},
+                "api": ("per rank: pinned host images -> pm_error_matrix rows -> pm_local_search_sharded_async -> "
+                        "pm_cost_sharded_async -> pinned host r" if rows_layout else
+                        "per rank: pinned host images -> pm_error_matrix rows -> all-gather -> "
+                        "pm_local_search_multi_async -> pm_cost_async -> pinned host r")},
         "gpu_launches": launches,
         "roofline": dominant, "roofline_other": other,
         "breakdown_ms_rank0": part_ms,
@@ -522,7 +549,7 @@ def main():
     if world > 1:
         torch.cuda.set_device(local_rank)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    if (world > 1 and not args.independent) or args.sharded:
+    if (world > 1 and not args.independent) or args.sharded or args.e_layout == "rows":
         line, extra = bench_sharded(args, rank, world, local_rank)
     else:
         line, extra = bench_single(args, rank, world, local_rank)

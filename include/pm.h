@@ -205,6 +205,41 @@ pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int
                                            int32_t world, int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
                                            pm_stream_t stream);
 
+/* Multi-GPU Algorithm 2 over ROW-SHARDED E (the north_star
+ * layout): rank o holds only rows [h_row_begin[o], h_row_begin[o+1]) of E
+ * (e.g. its own pm_error_matrix row block), in a buffer mapped into every
+ * peer (d_E_peers[o] points at that shard's first row; leading dimension
+ * ld_E >= S elements, the same on every rank).  The protocol is that of
+ * pm_local_search_multi_async; the only difference is where E is read:
+ * each rank first writes the sigma-permuted copy of its own rows (reading
+ * R10's contiguous-run layout, DESIGN 6.1) into its workspace, and each
+ * TRAP tile then reads E[t][.] from the rank that owns row t, through
+ * NVLink peer loads -- no rank holds, gathers or replicates all of E.  Every
+ * round runs TRAP (no sparse rounds, which would need the whole matrix).
+ * Results are bit-identical to pm_local_search.
+ *   pm_trap_workspace_bytes_sharded : per-rank workspace size for S and
+ *            that rank's row count (the replicated-mode workspace followed
+ *            by its permuted rows); reset with pm_trap_workspace_reset.
+ *   pm_local_search_sharded_async : this rank's part.  h_row_begin : host
+ *            int32 [world+1], 0 = h_row_begin[0] <= ... <= h_row_begin[world]
+ *            = S, identical on every rank; d_E_peers, d_perm_peers,
+ *            d_ws_peers : host arrays of `world` device pointers (a rank
+ *            with no rows may pass NULL for its shard).  All ranks must run
+ *            concurrently; every wait is bounded as above.
+ *   pm_local_search_sharded_emulated : test hook -- E is split evenly into
+ *            `world` separate shard buffers on the current device and all
+ *            ranks run in one launch; d_perm in/out as pm_local_search.
+ * Unsupported shapes: as pm_local_search_multi_async (PM_ERR_UNSUPPORTED
+ * before anything is enqueued); bad pointers / row bounds: PM_ERR_INVALID. */
+size_t pm_trap_workspace_bytes_sharded(int32_t S, int32_t rows);
+pm_status_t pm_local_search_sharded_async(const int32_t* const* d_E_peers, const int32_t* h_row_begin, int64_t ld_E,
+                                          int32_t S, int32_t* const* d_perm_peers, void* const* d_ws_peers,
+                                          int32_t rank, int32_t world, int32_t max_rounds, int64_t* d_result,
+                                          pm_stream_t stream);
+pm_status_t pm_local_search_sharded_emulated(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                             int32_t world, int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
+                                             pm_stream_t stream);
+
 /* The method PM_LS_AUTO selects for S on the current device (host-only). */
 int32_t pm_ls_auto_method(int32_t S);
 
@@ -220,6 +255,15 @@ pm_status_t pm_cost(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* 
 /* Eq. (2) without the host sync: d_cost (int64 [1], device) is overwritten. */
 pm_status_t pm_cost_async(const int32_t* d_E, int64_t ld_E, int32_t S, const int32_t* d_perm,
                           int64_t* d_cost, pm_stream_t stream);
+
+/* Eq. (2) over ROW-SHARDED E (the layout of pm_local_search_sharded_async):
+ * d_E_peers / h_row_begin / world / ld_E as there (peer-mapped shards, host
+ * arrays); d_perm int32 [S] on this device; d_cost (int64 [1], device) is
+ * overwritten with sum_u E[r[u]][u], each term read from the shard owning row
+ * r[u].  Async on stream; PM_ERR_INVALID on bad pointers or bounds. */
+pm_status_t pm_cost_sharded_async(const int32_t* const* d_E_peers, const int32_t* h_row_begin, int32_t world,
+                                  int64_t ld_E, int32_t S, const int32_t* d_perm, int64_t* d_cost,
+                                  pm_stream_t stream);
 
 /* The whole approximation pipeline of Sec. V in one call, on
  * device buffers: Step 1 + Step 2 into d_E (caller-owned, [S][ld_E]), r :=

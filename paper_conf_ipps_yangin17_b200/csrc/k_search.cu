@@ -271,8 +271,8 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
 }
 
 // ------------------------------------------------------------ Eq. (2) ----
-__global__ void __launch_bounds__(256) k_cost(const int32_t* __restrict__ E, int64_t ld, int32_t S,
-                                              const int32_t* __restrict__ perm,
+template <class Rows>
+__global__ void __launch_bounds__(256) k_cost(const Rows E, int32_t S, const int32_t* __restrict__ perm,
                                               unsigned long long* __restrict__ cost) {
   // up to 8 gathers per thread, all r loads then all E loads in flight (two
   // memory round trips instead of one per gather)
@@ -285,7 +285,7 @@ __global__ void __launch_bounds__(256) k_cost(const int32_t* __restrict__ E, int
     for (int q = 0; q < U; ++q) rq[q] = (u0 + q * stride < S) ? __ldg(perm + u0 + q * stride) : -1;
 #pragma unroll
     for (int q = 0; q < U; ++q)
-      if (rq[q] >= 0) s += __ldg(E + (int64_t)rq[q] * ld + (u0 + q * stride));
+      if (rq[q] >= 0) s += __ldg(E(rq[q]) + (u0 + q * stride));
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
@@ -300,8 +300,9 @@ __global__ void __launch_bounds__(256) k_cost(const int32_t* __restrict__ E, int
   }
 }
 
-cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm, int64_t* d_cost,
-                        cudaStream_t st) {
+template <class Rows>
+static cudaError_t launch_cost_rows(const Rows& E, int32_t S, const int32_t* perm, int64_t* d_cost,
+                                    cudaStream_t st) {
   int blocks = (S + 2047) / 2048;   // <= 8 gathers per thread
   if (blocks < 1) blocks = 1;
   if (blocks > 148) blocks = 148;
@@ -309,9 +310,19 @@ cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t*
     cudaError_t e = cudaMemsetAsync(d_cost, 0, sizeof(int64_t), st);
     if (e != cudaSuccess) return e;
   }
-  k_cost<<<blocks, 256, 0, st>>>(E, ldE, S, perm, reinterpret_cast<unsigned long long*>(d_cost));
+  k_cost<Rows><<<blocks, 256, 0, st>>>(E, S, perm, reinterpret_cast<unsigned long long*>(d_cost));
   note_launch();
   return cudaGetLastError();
+}
+
+cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm, int64_t* d_cost,
+                        cudaStream_t st) {
+  return launch_cost_rows(PlainRows{E, ldE}, S, perm, d_cost, st);
+}
+
+cudaError_t launch_cost_sharded(const ShardRows& rows, int32_t S, const int32_t* perm, int64_t* d_cost,
+                                cudaStream_t st) {
+  return launch_cost_rows(rows, S, perm, d_cost, st);
 }
 
 }  // namespace pm

@@ -50,6 +50,7 @@
 
 #include <atomic>
 #include <cstdio>
+#include <type_traits>
 #include <cstdlib>
 
 #include "pm_internal.cuh"
@@ -208,6 +209,7 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* mbar, uint32_t parity
 // (first slots), j < nA + nB -> slot u0 - (a2 + j - nA) (second slots),
 // j = nA + nB -> S - 1 (only when a == 0).  Pair k at step t (class c0 + t)
 // has slots u0 + t + k and u0 + t - k (or S - 1 for k = 0).
+
 struct TrapChunk {
   int32_t a, b, a2, nA, nB, Lc, K, m, Tp;
   __device__ __forceinline__ void local_slots(int32_t t, int32_t k, int32_t& j1, int32_t& j2) const {
@@ -234,18 +236,17 @@ struct TrapChunk {
 
 // One chunk of one phase: stage (state via `src`, E rows from global), replay
 // Tp classes.  Returns the swaps of the owned pairs.
-template <int PPL, int T, bool EP, typename Src>
+template <int PPL, int T, bool EP, typename Rows, typename Src>
 __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_t k1, int32_t c0, int32_t u0,
-                                          const int32_t* __restrict__ E, int64_t ld, int32_t S, Src src,
+                                          const Rows& erows, bool aligned, int32_t S, Src src,
                                           int4* s_st, int32_t* s_g, int32_t* s_E, int gt, int bar_id,
                                           bool vec, unsigned long long* tprof,
-                                          const int32_t* __restrict__ Ep, int64_t ldp, bool spec, bool coal) {
+                                          const Rows& eprows, bool spec, bool coal) {
   using SM = TrapSmem<PPL, T, EP>;
   static_assert(T <= 64, "one mask bit per class of a phase");
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
   const bool low = (C.a == 0);
-  const bool aligned = ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);
   int32_t* s_U = s_E + SM::UOFF;
   // ---- one thread per local slot j (= local tile j): its state, then its
   // tile's E row pieces, every copy independent of the others.  Both slots'
@@ -274,7 +275,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     // p0 = partner in class c0 (the fixed tile's runs are unused)
     const int32_t p0 = fx ? u0 : wrap_m(2 * c0 + 1 - x, m);
     const int32_t s0 = fx ? u0 : x;
-    const int32_t* row = E + (int64_t)g * ld;
+    const int32_t* row = erows(g);
     int32_t* dst = s_E + j * RS;
     if (EP) {
       // sigma-permuted rows: Ep[g][q] = E[g][2q mod m], so the stride-2 run
@@ -283,7 +284,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
       const int32_t ss = (int32_t)(((int64_t)s0 * ((m + 1) / 2)) % m);
       s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
                    : make_int4(j | (1 << 16), d, j * RS + (sp & 3), j * RS + SM::SP + (ss & 3) + 1);
-      const int32_t* prow = Ep + (int64_t)g * ldp;
+      const int32_t* prow = eprows(g);
       colA[i] = sp & ~3;
       colB[i] = ss & ~3;
       if (!coal) {
@@ -325,7 +326,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
         const int32_t cB = __shfl_sync(0xffffffffu, colB[i], sl);
         const int32_t js = wbase + sl + i * GT;
         if (js < Lc)
-          cp_async16(s_E + js * RS + ((r & 1) ? SM::SP : 0) + 4 * q, Ep + (int64_t)gr * ldp + ((r & 1) ? cB : cA) + 4 * q);
+          cp_async16(s_E + js * RS + ((r & 1) ? SM::SP : 0) + 4 * q, eprows(gr) + ((r & 1) ? cB : cA) + 4 * q);
       }
     }
   }
@@ -460,7 +461,9 @@ k_ls_trap(const TrapParams p) {
 
   const int32_t* __restrict__ E = p.E;
   const int64_t ld = p.ldE;
-  const bool vec = p.vec && ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);   // 16-byte row pieces
+  const bool aligned = ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);
+  const bool vec = p.vec && aligned;   // 16-byte row pieces
+  const PlainRows er{E, ld}, epr{p.Ep, p.ldp};
   const Classes cl(S);
   const int32_t m = cl.m, H = cl.half, K = cl.npairs - 1, ncls = cl.ncls;
   const int32_t W = p.W;
@@ -534,9 +537,9 @@ k_ls_trap(const TrapParams p) {
         if (have) {
           if (CLU) {
             const int2* rr = rep + cur * S;
-            mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
+            mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, er, aligned, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { const int2 v = rr[x]; g = v.x; d = v.y; el = -1; },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.coal);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, epr, spec, p.coal);
           } else {
             const int bi = p.nbsync ? (int)(qph % 3u) : cur;
             const int4* __restrict__ sc = bi == 0 ? p.sbuf[0] : (bi == 1 ? p.sbuf[1] : p.sbuf[2]);
@@ -557,11 +560,11 @@ k_ls_trap(const TrapParams p) {
               }
               group_sync(1 + grp, GT);
             }
-            mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
+            mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, er, aligned, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) {
                                          const int4 v = __ldcg(sc + x); g = v.x; d = v.y; el = v.z;
                                        },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, p.Ep, p.ldp, spec, p.coal);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, epr, spec, p.coal);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
           // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
@@ -906,7 +909,6 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
 // every rank's perm, so every rank returns the whole result.  The same
 // kernel runs all ranks inside one launch on one device for the test hook
 // pm_local_search_multi_emulated (peer pointers are then plain pointers).
-constexpr int kMaxRanks = 8;
 struct TrapRank {                 // one rank's workspace (see trap_ws_layout)
   int32_t* rbuf[3];
   int32_t* dbuf[3];
@@ -930,6 +932,10 @@ struct TrapMultiParams {
   int32_t spec;                   // speculative class steps
   int32_t coal;                   // coalesced staging of the Ep runs
   unsigned long long wait_ns;     // bound of every cross-rank wait
+  // E row-sharded across the ranks (SH kernels): row g of E and of Ep is read
+  // from its owner's shard (peer memory); no rank holds all of E
+  ShardRows esh, epsh;
+  int32_t sh_aligned;             // SH: every shard's rows are 16-byte aligned
 };
 
 __device__ __forceinline__ int32_t chunk_begin(int32_t r, int32_t nchunks, int32_t world) {
@@ -998,7 +1004,7 @@ __device__ __forceinline__ bool sys_barrier_arrive_wait(const TrapMultiParams& p
   return wait_ge_sys(p, r, p.rk[r].xbar, target);
 }
 
-template <int PPL, int T, bool EP>
+template <int PPL, int T, bool EP, bool SH>
 __global__ void __launch_bounds__(256, 1)
 k_ls_trap_mr(const TrapMultiParams p) {
   using SM = TrapSmem<PPL, T, EP>;
@@ -1021,7 +1027,18 @@ k_ls_trap_mr(const TrapMultiParams p) {
   const int32_t* __restrict__ E = me.E;
   const int64_t ld = p.ldE;
   const int32_t S = p.S;
-  const bool vec = p.vec && ((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0);
+  // p.vec: 16-byte row pieces allowed (the host checked the alignment of every shard)
+  const bool aligned = SH ? p.sh_aligned != 0 : (((ld & 3) == 0) && ((reinterpret_cast<uintptr_t>(E) & 15) == 0));
+  const bool vec = p.vec && aligned;
+  using Rows = typename std::conditional<SH, ShardRows, PlainRows>::type;
+  Rows er, epr;
+  if constexpr (SH) {
+    er = p.esh;
+    epr = p.epsh;
+  } else {
+    er = PlainRows{E, ld};
+    epr = PlainRows{me.Ep, p.ldp};
+  }
   const Classes cl(S);
   const int32_t m = cl.m, H = cl.half, K = cl.npairs - 1, ncls = cl.ncls;
   const int32_t W = p.W, world = p.world, nch = p.nchunks;
@@ -1031,18 +1048,32 @@ k_ls_trap_mr(const TrapMultiParams p) {
   if (p.out->status != PM_OK) return;   // uniform (written before launch)
 
   __shared__ int32_t s_abort, s_gab[8];   // s_gab[grp]: written by that group's thread 0 only
+  unsigned int xtarget = 0;
   if (threadIdx.x == 0) { s_cta_sw = 0; s_abort = 0; }
   if (gt == 0) s_gab[grp] = 0;
-  for (int32_t x = lb * blockDim.x + threadIdx.x; x < S; x += nloc * blockDim.x)
-    __stcg(me.dbuf[0] + x, __ldg(E + (int64_t)__ldcg(me.rbuf[0] + x) * ld + x));
+  bool ok = true;
+  if (SH) {
+    // every rank's E shard and its permuted rows were written before that
+    // rank's launch (stream order): after one cross-rank barrier every
+    // peer's shard is complete and may be read
+    __syncthreads();
+    if (leader) {
+      xtarget += (unsigned)world;
+      if (!sys_barrier_arrive_wait(p, r, xtarget)) s_abort = 1;
+    }
+    bar_target += nloc;
+    ok = grid_barrier_mr(p, r, me.bar, bar_target) && !s_abort;
+  }
+  if (ok)
+    for (int32_t x = lb * blockDim.x + threadIdx.x; x < S; x += nloc * blockDim.x)
+      __stcg(me.dbuf[0] + x, __ldg(er(__ldcg(me.rbuf[0] + x)) + x));
   bar_target += nloc;
-  bool ok = grid_barrier_mr(p, r, me.bar, bar_target);
+  ok = grid_barrier_mr(p, r, me.bar, bar_target) && ok;
 
   uint32_t q = 0;
   int32_t rounds = 0;
   int64_t total = 0;
   int status = PM_OK;
-  unsigned int xtarget = 0;
   int64_t prev_rs = -1;
   while (ok) {
     const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1);
@@ -1073,9 +1104,9 @@ k_ls_trap_mr(const TrapMultiParams p) {
           C.K = K; C.m = m; C.Tp = Tp;
           const int32_t* __restrict__ rc = me.rbuf[bi];
           const int32_t* __restrict__ dc = me.dbuf[bi];
-          mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, E, ld, S,
+          mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, er, aligned, S,
                                      [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { g = __ldcg(rc + x); d = __ldcg(dc + x); el = -1; },
-                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, me.Ep, p.ldp, spec, p.coal);
+                                     s_st, s_g, s_E, gt, 1 + grp, vec, nullptr, epr, spec, p.coal);
           // publish the owned slots to the ranks owning chunks ch-1, ch, ch+1
           int32_t own[3];
           int nown = 0;
@@ -1219,11 +1250,11 @@ static void trap_ws_layout(void* ws, int32_t S, int32_t* perm, const int32_t* E,
 size_t trap_ws_zero_bytes(int32_t S) { return 128 + sizeof(unsigned int) * ((size_t)S / 2 + 16); }
 
 // Launch `nloc` ranks [rank0, rank0 + nloc) of a world on the current device.
-template <int PPL, int T, bool EP>
+template <int PPL, int T, bool EP, bool SH = false>
 static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE,
                                      int32_t S, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
                                      int32_t max_log, cudaStream_t st, int32_t* handoff, int32_t sparse_T,
-                                     int64_t ldp) {
+                                     int64_t ldp, const ShardRows* esh = nullptr, const ShardRows* epsh = nullptr) {
   using SM = TrapSmem<PPL, T, EP>;
   if (S < ls_trap_min_S() || (S & 1) || world < 1 || world > kMaxRanks || nloc < 1) return PM_ERR_UNSUPPORTED;
   int dev = 0, nsm = 0, optin = 0;
@@ -1244,6 +1275,14 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   hp.wait_ns = (unsigned long long)knob("trap_wait_ms", 20000) * 1000000ull;
   hp.spec = knob("trap_spec", 1);
   hp.coal = knob("trap_coal", 1);
+  if (SH) {
+    hp.esh = *esh;
+    hp.epsh = *epsh;
+    bool al = (ldE & 3) == 0;
+    for (int o = 0; o < world; ++o) al = al && (reinterpret_cast<uintptr_t>(esh->base[o]) & 15) == 0;
+    hp.sh_aligned = al ? 1 : 0;
+    hp.vec = hp.vec && al;
+  }
   const int per_rank_chunks = (hp.nchunks + world - 1) / world;
   int cpc = (per_rank_chunks * nloc + nsm - 1) / nsm;
   int max_cpc = (int)((size_t)optin / SM::bytes);
@@ -1252,7 +1291,7 @@ static pm_status_t launch_trap_multi(TrapRank* ranks, int32_t world, int32_t ran
   if (cpc > max_cpc) cpc = max_cpc;
   const size_t smem = SM::bytes * cpc;
   const int threads = SM::X * cpc;
-  auto fn = k_ls_trap_mr<PPL, T, EP>;
+  auto fn = k_ls_trap_mr<PPL, T, EP, SH>;
   PM_CUDA_TRY(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int occ = 0;
   PM_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem));
@@ -1408,6 +1447,129 @@ pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* c
     sps.p = nullptr;
     return sparse_launch(&sr, st);
   }
+  return PM_OK;
+}
+
+// ---------------------------------------------------------------------
+// Row-sharded E (north_star's multi-GPU layout): rank o holds rows
+// [rb[o], rb[o+1]) of E, and builds the sigma-permuted copy of the same rows
+// into its workspace; every rank reads any tile's runs from the owner's
+// shard through peer memory, so no rank holds (or all-gathers) all of E.  No
+// sparse rounds (they would gather all of E): TRAP runs every round.
+static int64_t ep_ld(int32_t S) { return ((int64_t)S - 1 + 48 + 31) / 32 * 32; }
+static size_t ws_head_sharded(int32_t S) { return (trap_ws_bytes(S) + 255) / 256 * 256; }
+size_t trap_ws_bytes_sharded(int32_t S, int32_t rows) {
+  return ws_head_sharded(S) + sizeof(int32_t) * (size_t)rows * (size_t)ep_ld(S);
+}
+
+static pm_status_t check_shards(const int32_t* rb, int32_t S, int32_t world) {
+  if (world < 1 || world > kMaxRanks || !rb || rb[0] != 0 || rb[world] != S) return PM_ERR_INVALID;
+  for (int o = 0; o < world; ++o)
+    if (rb[o + 1] < rb[o]) return PM_ERR_INVALID;
+  return PM_OK;
+}
+
+static pm_status_t launch_sharded(TrapRank* ranks, int32_t world, int32_t rank0, int32_t nloc, int64_t ldE,
+                                  int32_t S, int32_t max_rounds, LsResult* dev_out, int64_t* dev_per_round,
+                                  int32_t max_log, cudaStream_t st, const ShardRows& esh, const ShardRows& epsh) {
+  const int64_t ldp = epsh.ld;
+  const int32_t v = trap_multi_variant(S, ldE);
+  if (v == 6)
+    return launch_trap_multi<6, 48, true, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                                max_log, st, nullptr, 0, ldp, &esh, &epsh);
+  if (v == 5)
+    return launch_trap_multi<4, 32, true, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                                max_log, st, nullptr, 0, ldp, &esh, &epsh);
+  return launch_trap_multi<2, 16, true, true>(ranks, world, rank0, nloc, ldE, S, max_rounds, dev_out, dev_per_round,
+                                              max_log, st, nullptr, 0, ldp, &esh, &epsh);
+}
+
+pm_status_t trap_multi_rank_sharded(const int32_t* const* E_peers, const int32_t* rb, int64_t ldE, int32_t S,
+                                    int32_t* const* perm_peers, void* const* ws_peers, int32_t rank, int32_t world,
+                                    int32_t max_rounds, LsResult* dev_out, cudaStream_t st) {
+  {
+    const pm_status_t v = check_shards(rb, S, world);
+    if (v != PM_OK) return v;
+    if (rank < 0 || rank >= world) return PM_ERR_INVALID;
+    const pm_status_t w = trap_multi_supported(S, ldE, world);
+    if (w != PM_OK) return w;
+  }
+  PM_CUDA_TRY(launch_perm_check(perm_peers[rank], S, dev_out, st));
+  const size_t head = ws_head_sharded(S);
+  const int64_t ldp = ep_ld(S);
+  ShardRows esh = {}, epsh = {};
+  esh.world = epsh.world = world;
+  esh.ld = ldE;
+  epsh.ld = ldp;
+  TrapRank ranks[kMaxRanks];
+  for (int o = 0; o < world; ++o) {
+    trap_ws_layout(ws_peers[o], S, perm_peers[o], nullptr, ranks[o]);
+    esh.base[o] = E_peers[o];
+    epsh.base[o] = reinterpret_cast<const int32_t*>(static_cast<const char*>(ws_peers[o]) + head);
+  }
+  for (int o = 0; o <= world; ++o) esh.rb[o] = epsh.rb[o] = rb[o];
+  // this rank's rows of Ep, into its own workspace (peers read them after
+  // the kernel's opening cross-rank barrier)
+  const int32_t rows = rb[rank + 1] - rb[rank];
+  if (rows > 0)
+    PM_CUDA_TRY(launch_permute_cols(E_peers[rank], ldE, const_cast<int32_t*>(epsh.base[rank]), ldp, rows, S - 1, 48,
+                                    st));
+  return launch_sharded(ranks, world, rank, 1, ldE, S, max_rounds, dev_out, nullptr, 0, st, esh, epsh);
+}
+
+// Every rank of a world in one launch on the current device (test hook): E's
+// rows copied into `world` separate shard buffers, each with its own Ep rows.
+pm_status_t trap_multi_emulated_sharded(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
+                                        int32_t max_rounds, LsResult* dev_out, cudaStream_t st) {
+  {
+    const pm_status_t w = trap_multi_supported(S, ldE, world);
+    if (w != PM_OK) return w;
+  }
+  PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
+  int32_t rb[kMaxRanks + 1];
+  for (int o = 0; o <= world; ++o) rb[o] = (int32_t)(((int64_t)S * o) / world);
+  const size_t head = ws_head_sharded(S);
+  const int64_t ldp = ep_ld(S);
+  const size_t pb = ((size_t)S * sizeof(int32_t) + 255) / 256 * 256;
+  size_t total = 0;
+  size_t off_ws[kMaxRanks], off_perm[kMaxRanks], off_e[kMaxRanks];
+  for (int o = 0; o < world; ++o) {
+    const int32_t rows = rb[o + 1] - rb[o];
+    off_ws[o] = total;
+    total += (trap_ws_bytes_sharded(S, rows) + 255) / 256 * 256;
+    off_perm[o] = total;
+    total += pb;
+    off_e[o] = total;
+    total += ((size_t)rows * (size_t)ldE * sizeof(int32_t) + 255) / 256 * 256;
+  }
+  ScopedScratch buf(st);
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, total, st));
+  char* b = buf.as<char>();
+  ShardRows esh = {}, epsh = {};
+  esh.world = epsh.world = world;
+  esh.ld = ldE;
+  epsh.ld = ldp;
+  TrapRank ranks[kMaxRanks];
+  for (int o = 0; o < world; ++o) {
+    const int32_t rows = rb[o + 1] - rb[o];
+    void* ws = b + off_ws[o];
+    int32_t* pr = reinterpret_cast<int32_t*>(b + off_perm[o]);
+    int32_t* es = reinterpret_cast<int32_t*>(b + off_e[o]);
+    PM_CUDA_TRY(cudaMemsetAsync(ws, 0, trap_ws_zero_bytes(S), st));
+    PM_CUDA_TRY(cudaMemcpyAsync(pr, perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
+    if (rows > 0)
+      PM_CUDA_TRY(cudaMemcpy2DAsync(es, sizeof(int32_t) * ldE, E + (int64_t)rb[o] * ldE, sizeof(int32_t) * ldE,
+                                    sizeof(int32_t) * S, rows, cudaMemcpyDeviceToDevice, st));
+    trap_ws_layout(ws, S, pr, nullptr, ranks[o]);
+    esh.base[o] = es;
+    epsh.base[o] = reinterpret_cast<const int32_t*>(static_cast<char*>(ws) + head);
+    if (rows > 0)
+      PM_CUDA_TRY(launch_permute_cols(es, ldE, const_cast<int32_t*>(epsh.base[o]), ldp, rows, S - 1, 48, st));
+  }
+  for (int o = 0; o <= world; ++o) esh.rb[o] = epsh.rb[o] = rb[o];
+  const pm_status_t s = launch_sharded(ranks, world, 0, world, ldE, S, max_rounds, dev_out, nullptr, 0, st, esh, epsh);
+  if (s != PM_OK) return s;
+  PM_CUDA_TRY(cudaMemcpyAsync(perm, ranks[world - 1].perm, sizeof(int32_t) * S, cudaMemcpyDeviceToDevice, st));
   return PM_OK;
 }
 }  // namespace pm

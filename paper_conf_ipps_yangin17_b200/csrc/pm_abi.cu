@@ -343,6 +343,56 @@ pm_status_t pm_local_search_multi_emulated(const int32_t* d_E, int64_t ld_E, int
   return (pm_status_t)h.status;
 }
 
+size_t pm_trap_workspace_bytes_sharded(int32_t S, int32_t rows) {
+  return (S < 2 || rows < 0 || rows > S) ? 0 : trap_ws_bytes_sharded(S, rows);
+}
+
+pm_status_t pm_local_search_sharded_async(const int32_t* const* d_E_peers, const int32_t* h_row_begin, int64_t ld_E,
+                                          int32_t S, int32_t* const* d_perm_peers, void* const* d_ws_peers,
+                                          int32_t rank, int32_t world, int32_t max_rounds, int64_t* d_result,
+                                          pm_stream_t stream) {
+  if (!d_E_peers || !h_row_begin || !d_perm_peers || !d_ws_peers || !d_result || ld_E < S || max_rounds < 0)
+    return PM_ERR_INVALID;
+  if (world < 1 || world > 8 || rank < 0 || rank >= world) return PM_ERR_INVALID;
+  if (h_row_begin[0] != 0 || h_row_begin[world] != S) return PM_ERR_INVALID;
+  for (int r = 0; r < world; ++r) {
+    if (!d_perm_peers[r] || !d_ws_peers[r] || h_row_begin[r + 1] < h_row_begin[r]) return PM_ERR_INVALID;
+    if (!d_E_peers[r] && h_row_begin[r + 1] > h_row_begin[r]) return PM_ERR_INVALID;
+  }
+  {
+    const pm_status_t v = trap_multi_supported(S, ld_E, world);
+    if (v != PM_OK) return v;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
+  return trap_multi_rank_sharded(d_E_peers, h_row_begin, ld_E, S, d_perm_peers, d_ws_peers, rank, world, max_rounds,
+                                 reinterpret_cast<LsResult*>(d_result), st);
+}
+
+pm_status_t pm_local_search_sharded_emulated(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                             int32_t world, int32_t max_rounds, int32_t* h_rounds, int64_t* h_swaps,
+                                             pm_stream_t stream) {
+  if (!d_E || !d_perm || ld_E < S || max_rounds < 0 || world < 1 || world > 8) return PM_ERR_INVALID;
+  {
+    const pm_status_t v = trap_multi_supported(S, ld_E, world);
+    if (v != PM_OK) return v;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  DevBuf buf;
+  buf.st = st;
+  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, sizeof(LsResult), st));
+  LsResult* dres = reinterpret_cast<LsResult*>(buf.p);
+  PM_CUDA_TRY(cudaMemsetAsync(dres, 0, sizeof(LsResult), st));
+  pm_status_t s = trap_multi_emulated_sharded(d_E, ld_E, S, d_perm, world, max_rounds, dres, st);
+  if (s != PM_OK) return s;
+  LsResult h;
+  PM_CUDA_TRY(cudaMemcpyAsync(&h, dres, sizeof(h), cudaMemcpyDeviceToHost, st));
+  PM_CUDA_TRY(cudaStreamSynchronize(st));
+  if (h_rounds) *h_rounds = (int32_t)h.rounds;
+  if (h_swaps) *h_swaps = h.swaps;
+  return (pm_status_t)h.status;
+}
+
 int32_t pm_ls_auto_method(int32_t S) {
   // measured on B200 (whole search incl. sparse rounds): TRAP for
   // even S >= 256 (config 1/2/3/4: 0.42/1.50/10.7/111 ms against WINDOW
@@ -356,6 +406,24 @@ pm_status_t pm_cost_async(const int32_t* d_E, int64_t ld_E, int32_t S, const int
                           pm_stream_t stream) {
   if (!d_E || !d_perm || !d_cost || S < 1 || ld_E < S) return PM_ERR_INVALID;
   PM_CUDA_TRY(launch_cost(d_E, ld_E, S, d_perm, d_cost, (cudaStream_t)stream));
+  return PM_OK;
+}
+
+pm_status_t pm_cost_sharded_async(const int32_t* const* d_E_peers, const int32_t* h_row_begin, int32_t world,
+                                  int64_t ld_E, int32_t S, const int32_t* d_perm, int64_t* d_cost,
+                                  pm_stream_t stream) {
+  if (!d_E_peers || !h_row_begin || !d_perm || !d_cost || S < 1 || ld_E < S) return PM_ERR_INVALID;
+  if (world < 1 || world > kMaxRanks || h_row_begin[0] != 0 || h_row_begin[world] != S) return PM_ERR_INVALID;
+  ShardRows rows = {};
+  rows.world = world;
+  rows.ld = ld_E;
+  for (int o = 0; o < world; ++o) {
+    if (h_row_begin[o + 1] < h_row_begin[o]) return PM_ERR_INVALID;
+    if (!d_E_peers[o] && h_row_begin[o + 1] > h_row_begin[o]) return PM_ERR_INVALID;
+    rows.base[o] = d_E_peers[o];
+  }
+  for (int o = 0; o <= world; ++o) rows.rb[o] = h_row_begin[o];
+  PM_CUDA_TRY(launch_cost_sharded(rows, S, d_perm, d_cost, (cudaStream_t)stream));
   return PM_OK;
 }
 

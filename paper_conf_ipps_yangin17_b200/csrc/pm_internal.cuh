@@ -133,8 +133,34 @@ cudaError_t launch_permute_cols(const int32_t* E, int64_t ldE, int32_t* Ep, int6
 pm_status_t run_window(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                        LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
                        int32_t* handoff = nullptr, int32_t sparse_T = 0);
-cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm,
-                        int64_t* d_cost, cudaStream_t st);
+constexpr int kMaxRanks = 8;
+
+// Where row g of E (or of its sigma-permuted copy) lives: one matrix, or
+// row shards across the ranks of a multi-GPU world (rank o holds rows
+// [rb[o], rb[o+1]) at base[o], a peer pointer).
+struct PlainRows {
+  const int32_t* base;
+  int64_t ld;
+  __device__ __forceinline__ const int32_t* operator()(int32_t g) const { return base + (int64_t)g * ld; }
+};
+struct ShardRows {
+  const int32_t* base[kMaxRanks];
+  int32_t rb[kMaxRanks + 1];
+  int32_t world;
+  int64_t ld;
+  __device__ __forceinline__ const int32_t* operator()(int32_t g) const {
+    int o = 0;
+    while (o + 1 < world && g >= rb[o + 1]) ++o;
+    return base[o] + (int64_t)(g - rb[o]) * ld;
+  }
+};
+
+cudaError_t launch_cost(const int32_t* E, int64_t ldE, int32_t S, const int32_t* perm, int64_t* d_cost,
+                        cudaStream_t st);
+// Eq. (2) over row-sharded E (peer-mapped shards)
+cudaError_t launch_cost_sharded(const ShardRows& rows, int32_t S, const int32_t* perm, int64_t* d_cost,
+                                cudaStream_t st);
+
 // ---- sparse rounds (k_sparse.cu): quiet rounds of Alg. 2 ----
 struct SpParams {
   const int32_t* E;
@@ -206,6 +232,12 @@ pm_status_t trap_multi_emulated(const int32_t* E, int64_t ldE, int32_t S, int32_
 pm_status_t trap_multi_rank(const int32_t* E, int64_t ldE, int32_t S, int32_t* const* perm_peers,
                             void* const* ws_peers, int32_t rank, int32_t world, int32_t max_rounds,
                             LsResult* dev_out, int64_t* dev_per_round, int32_t max_log, cudaStream_t st);
+size_t trap_ws_bytes_sharded(int32_t S, int32_t rows);
+pm_status_t trap_multi_rank_sharded(const int32_t* const* E_peers, const int32_t* rb, int64_t ldE, int32_t S,
+                                    int32_t* const* perm_peers, void* const* ws_peers, int32_t rank, int32_t world,
+                                    int32_t max_rounds, LsResult* dev_out, cudaStream_t st);
+pm_status_t trap_multi_emulated_sharded(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t world,
+                                        int32_t max_rounds, LsResult* dev_out, cudaStream_t st);
 
 // Histogram matching of I to T (k_hist.cu, reading R12).
 int32_t hist_max_channels();

@@ -2,14 +2,16 @@
 
 Step 2 (the error matrix, Eq. 1) shards naturally by input-tile rows:
 rank g computes rows [row_begin, row_end) of E against all S target tiles
-(`pm_error_matrix(row_begin, row_end)`, no exchange).  Algorithm 2 does not
-shard (every colour class is a global perfect matching), so a
-job either
+(`pm_error_matrix(row_begin, row_end)`, no exchange).  Algorithm 2's colour
+classes are global perfect matchings, so the search itself is
+one job across the ranks, exchanging chunk-boundary slots over peer memory:
 
-* runs independent photomosaics, one per rank (the benchmark: weak scaling,
-  no data-path collective), or
-* computes E row-sharded and all-gathers it when every rank needs the full
-  matrix (`error_matrix_sharded(..., gather=True)`).
+* `local_search_multi`: every rank holds all of E (gathered with
+  `error_matrix_sharded(..., gather=True)`), sparse rounds included;
+* `photomosaic_sharded` / `local_search_sharded`: E stays row-sharded in
+  symmetric memory and every rank reads the rows it needs from their owner
+  over NVLink (no rank holds all of E: the layout for matrices larger than
+  one GPU).
 
 Everything here is host-side marshalling around `pm` calls and
 torch.distributed collectives; no compute happens in Python.
@@ -111,3 +113,81 @@ def local_search_multi(E: torch.Tensor, perm: torch.Tensor | None = None, max_ro
         perm.copy_(out)
         out = perm
     return out, rounds, swaps
+
+
+def _symm_alloc(nbytes: int, device, group):
+    import torch.distributed._symmetric_memory as symm_mem
+    buf = symm_mem.empty(nbytes, dtype=torch.uint8, device=device)
+    hdl = symm_mem.rendezvous(buf, (group or dist.group.WORLD).group_name)
+    return buf, [int(p) for p in hdl.buffer_ptrs]
+
+
+def _sharded_layout(S: int, world: int):
+    from . import pm
+    bounds = [shard_rows(S, world, g) for g in range(world)]
+    rows_max = max(e - b for b, e in bounds)
+    ws = (pm.trap_workspace_bytes_sharded(S, rows_max) + 255) // 256 * 256
+    pb = (4 * S + 255) // 256 * 256
+    return [b for b, _ in bounds] + [S], rows_max, ws, pb
+
+
+def _run_sharded(buf, ptrs, S: int, perm, max_rounds: int, group):
+    from . import pm
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    rb, rows_max, ws, pb = _sharded_layout(S, world)
+    my_perm = buf[ws:ws + 4 * S].view(torch.int32)
+    my_perm.copy_(torch.arange(S, dtype=torch.int32, device=buf.device) if perm is None else perm)
+    buf[:ws].zero_()
+    torch.cuda.synchronize(buf.device)
+    dist.barrier(group)                                   # every workspace reset, every shard written
+    result = torch.zeros(3, dtype=torch.int64, device=buf.device)
+    pm.local_search_sharded_async([p + ws + pb for p in ptrs], rb, S, S, [p + ws for p in ptrs], ptrs, rank, world,
+                                  result, max_rounds=max_rounds)
+    torch.cuda.synchronize(buf.device)
+    dist.barrier(group)                                   # no rank frees its buffer while peers may read it
+    status, rounds, swaps = (int(v) for v in result.tolist())
+    if status not in (0, 3):
+        raise pm.PMError(status, "pm_local_search_sharded_async")
+    out = my_perm.clone()
+    if perm is not None:
+        perm.copy_(out)
+        out = perm
+    return out, rounds, swaps
+
+
+def local_search_sharded(E_part: torch.Tensor, S: int, perm: torch.Tensor | None = None, max_rounds: int = 0,
+                         group=None):
+    """Algorithm 2 across the ranks over ROW-SHARDED E with
+    pm_local_search_sharded_async: E_part = this rank's rows
+    shard_rows(S, world, rank) of E (e.g. error_matrix_sharded's part).  The
+    shard is copied into symmetric memory next to the workspace and perm;
+    every rank returns the final r.  Returns (perm, rounds, swaps)."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    rb, rows_max, ws, pb = _sharded_layout(S, world)
+    b, e = rb[rank], rb[rank + 1]
+    if tuple(E_part.shape) != (e - b, S):
+        raise ValueError(f"rank {rank} expects E rows [{b}, {e}) x {S}, got {tuple(E_part.shape)}")
+    buf, ptrs = _symm_alloc(ws + pb + 4 * rows_max * S, E_part.device, group)
+    buf[ws + pb:ws + pb + 4 * (e - b) * S].view(torch.int32).view(e - b, S).copy_(E_part)
+    return _run_sharded(buf, ptrs, S, perm, max_rounds, group)
+
+
+def photomosaic_sharded(I, T, M: int, perm: torch.Tensor | None = None, max_rounds: int = 0, group=None):
+    """Steps 2-3 across the ranks with E never gathered: rank g writes its
+    rows of E (pm_error_matrix) straight into its symmetric-memory shard,
+    then Algorithm 2 runs over the shards (local_search_sharded).  Returns
+    (perm, rounds, swaps)."""
+    from . import pm
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    N = I.shape[0]
+    S = (N // M) ** 2
+    rb, rows_max, ws, pb = _sharded_layout(S, world)
+    b, e = rb[rank], rb[rank + 1]
+    buf, ptrs = _symm_alloc(ws + pb + 4 * rows_max * S, I.device, group)
+    if e > b:
+        pm.error_matrix(I, T, M, rows=(b, e), out=buf[ws + pb:ws + pb + 4 * (e - b) * S].view(torch.int32).view(e - b, S))
+    return _run_sharded(buf, ptrs, S, perm, max_rounds, group)
+

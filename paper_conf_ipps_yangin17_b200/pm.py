@@ -54,6 +54,10 @@ _SIGS = [
     ("pm_trap_workspace_reset", ctypes.c_int, [_P, _I32, _P]),
     ("pm_local_search_multi_async", ctypes.c_int, [_P, _I64, _I32, _P, _P, _I32, _I32, _I32, _P, _P]),
     ("pm_local_search_multi_emulated", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P]),
+    ("pm_trap_workspace_bytes_sharded", ctypes.c_size_t, [_I32, _I32]),
+    ("pm_local_search_sharded_async", ctypes.c_int, [_P, _P, _I64, _I32, _P, _P, _I32, _I32, _I32, _P, _P]),
+    ("pm_cost_sharded_async", ctypes.c_int, [_P, _P, _I32, _I64, _I32, _P, _P, _P]),
+    ("pm_local_search_sharded_emulated", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P]),
     ("pm_tuning_set", ctypes.c_int, [ctypes.c_char_p, _I32]),
     ("pm_tuning_reset", None, []),
     ("pm_scratch_trim", ctypes.c_int, []),
@@ -252,6 +256,39 @@ def local_search_multi_async(E, perm_ptrs, ws_ptrs, rank: int, world: int, resul
            "pm_local_search_multi_async")
 
 
+def local_search_sharded_emulated(E, world: int, perm=None, max_rounds: int = 0, stream=None):
+    """pm_local_search_sharded_emulated (test hook): the row-sharded multi-GPU
+    search with `world` ranks (E split into `world` shard buffers) in one
+    launch on this device.  Returns (perm, rounds, swaps)."""
+    torch = _torch()
+    _dev(E, torch.int32)
+    S = E.shape[0]
+    if perm is None:
+        perm = torch.arange(S, dtype=torch.int32, device=E.device)
+    rounds, swaps = ctypes.c_int32(0), ctypes.c_int64(0)
+    _check(lib().pm_local_search_sharded_emulated(E.data_ptr(), E.stride(0), S, perm.data_ptr(), world, max_rounds,
+                                                  ctypes.byref(rounds), ctypes.byref(swaps), _stream(stream)),
+           "pm_local_search_sharded_emulated", (PM_OK, PM_ERR_NOT_CONVERGED))
+    return perm, int(rounds.value), int(swaps.value)
+
+
+def trap_workspace_bytes_sharded(S: int, rows: int) -> int:
+    return int(lib().pm_trap_workspace_bytes_sharded(S, rows))
+
+
+def local_search_sharded_async(E_ptrs, row_begin, ld_E: int, S: int, perm_ptrs, ws_ptrs, rank: int, world: int,
+                               result, max_rounds: int = 0, stream=None):
+    """pm_local_search_sharded_async: this rank's part of the search over
+    row-sharded E; E_ptrs / perm_ptrs / ws_ptrs = every rank's shard / perm /
+    workspace device pointers as mapped into this process (ints), row_begin
+    the world+1 shard bounds."""
+    P = ctypes.c_void_p * world
+    RB = ctypes.c_int32 * (world + 1)
+    _check(lib().pm_local_search_sharded_async(P(*E_ptrs), RB(*row_begin), ld_E, S, P(*perm_ptrs), P(*ws_ptrs),
+                                               rank, world, max_rounds, result.data_ptr(), _stream(stream)),
+           "pm_local_search_sharded_async")
+
+
 def ls_auto_method(S: int) -> str:
     """Name of the method PM_LS_AUTO picks for S on the current device."""
     code = int(lib().pm_ls_auto_method(S))
@@ -277,6 +314,15 @@ def cost_async(E, perm, out, stream=None):
 
 
 # ------------------------------------------------------- whole pipeline ----
+def cost_sharded_async(E_ptrs, row_begin, ld_E: int, S: int, perm, out, stream=None):
+    """pm_cost_sharded_async: Eq. (2) over row-sharded E (peer pointers)."""
+    world = len(E_ptrs)
+    P = ctypes.c_void_p * world
+    RB = ctypes.c_int32 * (world + 1)
+    _check(lib().pm_cost_sharded_async(P(*E_ptrs), RB(*row_begin), world, ld_E, S, perm.data_ptr(), out.data_ptr(),
+                                       _stream(stream)), "pm_cost_sharded_async")
+
+
 def photomosaic(I, T, M: int, method: str = "auto", E=None, perm=None, stream=None):
     """pm_photomosaic on device images: returns (perm, rounds, swaps, cost, E)."""
     torch = _torch()

@@ -135,3 +135,45 @@ def test_multi_rank_entry_points_validate_before_any_launch(pm):
     assert L.pm_local_search_multi_async(fake, S, S, P2(fake, None), P2(fake, fake), 0, 2, 0, fake, None) == pm.PM_ERR_INVALID
     assert L.pm_trap_workspace_reset(None, S, None) == pm.PM_ERR_INVALID
     assert L.pm_local_search_multi_emulated(None, S, S, fake, 2, 0, None, None, None) == pm.PM_ERR_INVALID
+
+
+def test_sharded_entry_points_validate_before_any_launch(pm):
+    # host-side checks of the row-sharded multi-GPU boundary (no device needed)
+    import ctypes
+    L = pm.lib()
+    S = 1024
+    full = pm.trap_workspace_bytes(S)
+    half = pm.trap_workspace_bytes_sharded(S, S // 2)
+    assert half >= full + 4 * (S // 2) * (S - 1)          # + this rank's permuted rows
+    assert pm.trap_workspace_bytes_sharded(S, S) > half
+    assert pm.trap_workspace_bytes_sharded(S, S + 1) == 0 and pm.trap_workspace_bytes_sharded(S, -1) == 0
+    P2 = ctypes.c_void_p * 2
+    RB = ctypes.c_int32 * 3
+    fake = 0x1000
+    ok = (P2(fake, fake), RB(0, S // 2, S), S, S, P2(fake, fake), P2(fake, fake), 0, 2, 0, fake, None)
+
+    def call(**kw):
+        a = list(ok)
+        for i, v in kw.items():
+            a[int(i[1:])] = v
+        return L.pm_local_search_sharded_async(*a)
+
+    assert call(a0=None) == pm.PM_ERR_INVALID                       # no shard table
+    assert call(a1=None) == pm.PM_ERR_INVALID                       # no row bounds
+    assert call(a1=RB(0, S // 2, S - 2)) == pm.PM_ERR_INVALID       # bounds do not end at S
+    assert call(a1=RB(1, S // 2, S)) == pm.PM_ERR_INVALID           # ... nor start at 0
+    assert call(a1=RB(0, S, S // 2)) == pm.PM_ERR_INVALID           # decreasing
+    assert call(a0=P2(fake, None)) == pm.PM_ERR_INVALID             # non-empty shard without a pointer
+    assert call(a2=S - 1) == pm.PM_ERR_INVALID                      # ld_E < S
+    assert call(a6=2) == pm.PM_ERR_INVALID                          # rank outside the world
+    assert call(a5=P2(fake, None)) == pm.PM_ERR_INVALID             # missing workspace
+    assert call(a9=None) == pm.PM_ERR_INVALID                       # no result
+    assert L.pm_local_search_sharded_emulated(None, S, S, fake, 2, 0, None, None, None) == pm.PM_ERR_INVALID
+    assert L.pm_local_search_sharded_emulated(fake, S, S, fake, 9, 0, None, None, None) == pm.PM_ERR_INVALID
+    C2 = ctypes.c_void_p * 2
+    assert L.pm_cost_sharded_async(None, RB(0, S // 2, S), 2, S, S, fake, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_cost_sharded_async(C2(fake, fake), RB(0, S // 2, S - 1), 2, S, S, fake, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_cost_sharded_async(C2(fake, None), RB(0, S // 2, S), 2, S, S, fake, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_cost_sharded_async(C2(fake, fake), RB(0, S // 2, S), 2, S - 1, S, fake, fake, None) == pm.PM_ERR_INVALID
+    assert L.pm_cost_sharded_async(C2(fake, fake), RB(0, S // 2, S), 9, S, S, fake, fake, None) == pm.PM_ERR_INVALID
+

@@ -674,6 +674,115 @@ def test_multi_rank_trap_symmetric_memory_world1():
             tdist.destroy_process_group()
 
 
+# ---- the same protocol over ROW-SHARDED E (pm_local_search_sharded_*): E's
+# rows split into `world` separate shard buffers, each rank's permuted rows in
+# its own workspace, every TRAP tile reading the owner's shard
+@pytest.mark.parametrize("N,M,fam,world", [(128, 8, "smooth", 2), (128, 8, "noise", 4), (512, 16, "smooth", 1),
+                                           (512, 16, "smooth", 2), (512, 16, "ties", 3), (512, 16, "smooth", 8),
+                                           (1024, 16, "smooth", 4), (1024, 16, "noise", 7),
+                                           (336, 8, "transposition", 5)])
+def test_sharded_trap_emulated(N, M, fam, world):
+    E_np = oracle_E(fam, N, M)
+    ref = oracle.local_search(E_np)
+    out, rounds, swaps = pm.local_search_sharded_emulated(dev(E_np), world)
+    assert (out.cpu().numpy() == ref[0]).all()
+    assert (rounds, swaps) == (ref[1], ref[2])
+
+
+@pytest.mark.parametrize("variant", ["0", "5", "6"])
+def test_sharded_trap_geometries(variant):
+    pm.tuning_set("trap_variant", int(variant))
+    E_np = oracle_E("smooth", 1024, 16)
+    ref = oracle.local_search(E_np)
+    out, rounds, swaps = pm.local_search_sharded_emulated(dev(E_np), 3)
+    assert (out.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+
+
+def test_sharded_trap_padded_ld_max_rounds_then_resume():
+    E_np = oracle_E("smooth", 512, 16)
+    S = E_np.shape[0]
+    big = torch.full((S, S + 5), -7, dtype=torch.int32, device=DEV)
+    big[:, :S] = dev(E_np)
+    ref = oracle.local_search(E_np, max_rounds=2)
+    out, rounds, swaps = pm.local_search_sharded_emulated(big[:, :S], 3, max_rounds=2)
+    assert (out.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+    ref2 = oracle.local_search(E_np, r0=ref[0])
+    out2, rounds2, swaps2 = pm.local_search_sharded_emulated(big[:, :S], 3, perm=out)
+    assert (out2.cpu().numpy() == ref2[0]).all() and (rounds2, swaps2) == (ref2[1], ref2[2])
+
+
+@pytest.mark.parametrize("bounds", ["even", "empty_first"])
+def test_sharded_async_one_process(bounds):
+    # pm_local_search_sharded_async itself at world 1 (own shard = all of E),
+    # and at world 2 with rank 1 owning every row while rank 0 holds none --
+    # rank 0 alone cannot finish, so that case is run as the bounded-wait
+    # failure path: PM_ERR_TIMEOUT, nothing hangs
+    E_np = oracle_E("smooth", 512, 16)
+    S = E_np.shape[0]
+    E = dev(E_np)
+    ref = oracle.local_search(E_np)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    if bounds == "even":
+        wsb = pm.trap_workspace_bytes_sharded(S, S)
+        ws = torch.zeros(wsb, dtype=torch.uint8, device=DEV)
+        perm = torch.arange(S, dtype=torch.int32, device=DEV)
+        pm.local_search_sharded_async([E.data_ptr()], [0, S], E.stride(0), S, [perm.data_ptr()], [ws.data_ptr()],
+                                      0, 1, res)
+        torch.cuda.synchronize()
+        assert int(res[0]) == pm.PM_OK
+        assert (perm.cpu().numpy() == ref[0]).all() and (int(res[1]), int(res[2])) == (ref[1], ref[2])
+    else:
+        wss = [torch.zeros(pm.trap_workspace_bytes_sharded(S, n), dtype=torch.uint8, device=DEV) for n in (0, S)]
+        perms = [torch.arange(S, dtype=torch.int32, device=DEV) for _ in range(2)]
+        with pm.tuning(trap_wait_ms=300):
+            pm.local_search_sharded_async([0, E.data_ptr()], [0, 0, S], E.stride(0), S,
+                                          [p_.data_ptr() for p_ in perms], [w.data_ptr() for w in wss], 0, 2, res)
+            torch.cuda.synchronize()
+        assert int(res[0]) == pm.PM_ERR_TIMEOUT
+        _check_ls(E_np, "trap")
+
+
+def test_sharded_symmetric_memory_world1():
+    # dist.photomosaic_sharded / local_search_sharded (symmetric-memory shard,
+    # workspace and perm; pm_error_matrix straight into the shard) at one rank
+    import torch.distributed as tdist
+
+    from paper_conf_ipps_yangin17_b200 import dist as pdist
+    I, T = pair("smooth", 512, 16)
+    E_np = oracle.error_matrix(I, T, 16)
+    ref = oracle.local_search(E_np)
+    own = not tdist.is_initialized()
+    if own:
+        tdist.init_process_group("nccl", init_method="tcp://127.0.0.1:29514", rank=0, world_size=1,
+                                 device_id=torch.device(DEV))
+    try:
+        try:
+            out, rounds, swaps = pdist.photomosaic_sharded(dev(I), dev(T), 16)
+        except (RuntimeError, AttributeError) as e:
+            pytest.skip(f"symmetric memory unavailable here: {e}")
+        assert (out.cpu().numpy() == ref[0]).all() and (rounds, swaps) == (ref[1], ref[2])
+        out2, rounds2, swaps2 = pdist.local_search_sharded(dev(E_np), E_np.shape[0])
+        assert (out2.cpu().numpy() == ref[0]).all() and (rounds2, swaps2) == (ref[1], ref[2])
+    finally:
+        if own:
+            tdist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_cost_sharded(world):
+    # Eq. (2) with E split into `world` separate shard buffers (uneven bounds)
+    E_np = oracle_E("noise", 512, 16)
+    S = E_np.shape[0]
+    rng = np.random.default_rng(world)
+    r = rng.permutation(S).astype(np.int32)
+    cuts = sorted(rng.integers(0, S + 1, size=world - 1).tolist())
+    rb = [0] + cuts + [S]
+    shards = [dev(E_np[rb[o]:rb[o + 1]]) if rb[o + 1] > rb[o] else None for o in range(world)]
+    out = torch.full((1,), -1, dtype=torch.int64, device=DEV)
+    pm.cost_sharded_async([0 if t is None else t.data_ptr() for t in shards], rb, S, S, dev(r), out)
+    assert int(out.item()) == oracle.cost(E_np, r)
+
+
 @pytest.mark.parametrize("coal", [0, 1])
 @pytest.mark.parametrize("ep,mode", [("0", "1"), ("0", "0"), ("1", "0"), ("1", "1")])
 def test_trap_sigma_permuted_and_plain_row_staging(ep, mode, coal):

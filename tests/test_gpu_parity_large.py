@@ -111,6 +111,14 @@ def test_cfg4_multi_rank_emulated_world8(cfg4):
     _assert_search((out, rounds, swaps, None, 0), ref, E_or, "config 4 world 8 (emulated)")
 
 
+def test_cfg4_sharded_emulated_world8(cfg4):
+    # E row-sharded over 8 ranks (separate shard buffers), read through the
+    # owner's shard: the whole search on TRAP rounds, same result
+    I, T, E_or, E_gpu, ref = cfg4
+    out, rounds, swaps = pm.local_search_sharded_emulated(E_gpu, 8)
+    _assert_search((out, rounds, swaps, None, 0), ref, E_or, "config 4 world 8 row-sharded (emulated)")
+
+
 def test_cfg4_max_rounds_then_resume(cfg4):
     I, T, E_or, E_gpu, ref = cfg4
     cut = oracle.local_search(E_or, max_rounds=3)
@@ -162,6 +170,13 @@ def test_cfg5_multi_rank_emulated_world8_first_rounds(cfg5):
     I, T, E_or, E_gpu, ref5 = cfg5
     out, rounds, swaps = pm.local_search_multi_emulated(E_gpu, 8, max_rounds=5)
     _assert_search((out, rounds, swaps, None, 3), ref5, E_or, "config 5 world 8 (emulated), 5 rounds")
+
+
+def test_cfg5_sharded_emulated_world8_first_rounds(cfg5):
+    # config 5's E (16 GiB) in 8 row shards of 2 GiB + their permuted copies
+    I, T, E_or, E_gpu, ref5 = cfg5
+    out, rounds, swaps = pm.local_search_sharded_emulated(E_gpu, 8, max_rounds=5)
+    _assert_search((out, rounds, swaps, None, 3), ref5, E_or, "config 5 world 8 row-sharded (emulated), 5 rounds")
 
 
 def test_cfg5_local_search_to_convergence(cfg5):

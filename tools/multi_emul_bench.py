@@ -1,6 +1,9 @@
 """Cost of the multi-GPU TRAP protocol on one GPU: pm_local_search_multi_emulated
 with every rank of a world in one launch (the GPU's SMs split among the ranks),
-against world = 1.  Development probe.  Usage: python tools/multi_emul_bench.py [cfgs] [worlds]"""
+against world = 1.  Development probe.  Usage:
+python tools/multi_emul_bench.py [cfgs] [worlds] [multi|sharded]
+(sharded: pm_local_search_sharded_emulated, E split into row-shard buffers;
+its time includes the shard copies and the permuted-row builds)"""
 import os
 import sys
 import time
@@ -15,6 +18,8 @@ _devknobs.apply(pm)
 
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["3", "4"])]
 worlds = [int(w) for w in (sys.argv[2].split(",") if len(sys.argv) > 2 else ["1", "2", "4", "8"])]
+mode = sys.argv[3] if len(sys.argv) > 3 else "multi"
+run = pm.local_search_sharded_emulated if mode == "sharded" else pm.local_search_multi_emulated
 for cfg in cfgs:
     c = synth.CONFIGS[cfg]
     I, T = synth.config_pair(cfg, "smooth", 0)
@@ -25,7 +30,7 @@ for cfg in cfgs:
         for rep in range(3):
             torch.cuda.synchronize()
             t0 = time.perf_counter()
-            perm, rounds, swaps = pm.local_search_multi_emulated(E, w)
+            perm, rounds, swaps = run(E, w)
             torch.cuda.synchronize()
             ts.append(time.perf_counter() - t0)
-        print(f"cfg{cfg} S={S} world={w} {min(ts) * 1e3:9.3f} ms rounds={rounds} swaps={swaps}", flush=True)
+        print(f"{mode} cfg{cfg} S={S} world={w} {min(ts) * 1e3:9.3f} ms rounds={rounds} swaps={swaps}", flush=True)
