@@ -13,6 +13,8 @@ import torch  # noqa: E402
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
 sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 import _devknobs  # noqa: E402
+if os.environ.get("PM_LIB"):   # a development build of the library (knockout experiments)
+    pm.LIB_PATH = os.environ["PM_LIB"]
 _devknobs.apply(pm)
 
 pm.tuning_set("trap_prof", int(os.environ.get("PM_TRAP_PROF", "1")))
@@ -26,7 +28,7 @@ for cfg in cfgs:
         perm = torch.arange(S, dtype=torch.int32, device="cuda")
         per = np.zeros(256, dtype=np.int64)
         r, sw = ctypes.c_int32(0), ctypes.c_int64(0)
-        st = pm.lib().pm_local_search_ex(E.data_ptr(), E.stride(0), S, perm.data_ptr(), 0, pm.METHODS["trap"],
+        st = pm.lib().pm_local_search_ex(E.data_ptr(), E.stride(0), S, perm.data_ptr(), int(os.environ.get("PM_MAX_ROUNDS", "0")), pm.METHODS["trap"],
                                          ctypes.byref(r), ctypes.byref(sw), per.ctypes.data, 256, None)
     ld, stp, bar, nph, pub, t0 = per[192:198]
     nph = max(int(nph), 1)
