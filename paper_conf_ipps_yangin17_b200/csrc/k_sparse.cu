@@ -112,8 +112,10 @@ __device__ __forceinline__ void scan_full_ep(const SpParams* __restrict__ p, int
       if (ok) {
         t = __ldg(r + y);
         dy = __ldg(d + y);
-        q = (int32_t)(((int64_t)c0 + H - (int64_t)y * H % m) % m);   // sigma-position of class c0's partner
-        q = q < 0 ? q + m : q;
+        // sigma-position of class c0's partner: c0 + H - sigma(y) mod m, where
+        // sigma(y) = y H mod m is y/2 or (y+m)/2 (m odd) -- no 64-bit remainder
+        q = c0 + H - ((y & 1) ? (y + m) >> 1 : y >> 1);
+        q = q < 0 ? q + m : (q >= m ? q - m : q);
       }
       int32_t val[32];
 #pragma unroll

@@ -127,6 +127,9 @@ __device__ __forceinline__ int32_t wrap_m(int32_t x, int32_t m) {
   return x >= m ? x - m : x;
 }
 
+// sigma(y) = y (m+1)/2 mod m for 0 <= y < m, m odd
+__device__ __forceinline__ int32_t sigma_m(int32_t y, int32_t m) { return (y & 1) ? (y + m) >> 1 : y >> 1; }
+
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -244,6 +247,7 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
                                           const Rows& eprows, bool spec, bool coal) {
   using SM = TrapSmem<PPL, T, EP>;
   static_assert(T <= 64, "one mask bit per class of a phase");
+  const unsigned long long t_in = tprof ? gtimer() : 0;   // trap_prof: tprof[1] issue, tprof[2] copy wait
   constexpr int RS = SM::RS, X = SM::X, GT = X;   // one pair position per thread
   const int32_t m = C.m, K = C.K, Tp = C.Tp, Lc = C.Lc;
   const bool low = (C.a == 0);
@@ -280,8 +284,11 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     if (EP) {
       // sigma-permuted rows: Ep[g][q] = E[g][2q mod m], so the stride-2 run
       // from column y is the contiguous run from q = sigma(y) = y (m+1)/2
-      const int32_t sp = (int32_t)(((int64_t)p0 * ((m + 1) / 2)) % m);
-      const int32_t ss = (int32_t)(((int64_t)s0 * ((m + 1) / 2)) % m);
+      // (m = S-1 is odd, so (m+1)/2 is the inverse of 2 mod m: sigma(y) = y/2
+      // for even y, (y+m)/2 for odd y -- no 64-bit remainder, which was four
+      // calls of the division routine per thread and phase)
+      const int32_t sp = sigma_m(p0, m);
+      const int32_t ss = sigma_m(s0, m);
       s_st[j] = fx ? make_int4(j | (1 << 16), d, SM::UOFF + ci * SM::NU + (u0 & 3), 0)
                    : make_int4(j | (1 << 16), d, j * RS + (sp & 3), j * RS + SM::SP + (ss & 3) + 1);
       const int32_t* prow = eprows(g);
@@ -306,34 +313,46 @@ __device__ __forceinline__ int trap_chunk(const TrapChunk& C, int32_t k0, int32_
     if (ci >= 0) stage_span(s_U + ci * SM::NU, row, u0 & ~3, SM::NU, m, aligned || vec);
   }
   if (EP && coal) {
-    // warp-cooperative copies of the runs of the warp's 32 slots: lane l of
-    // copy `ins` moves 16-byte piece P = 32 ins + l of the warp's 64 runs, so
-    // one warp instruction covers ~3.5 whole runs (contiguous pieces, ~18
-    // sectors / ~8 lines) instead of 32 pieces of 32 different runs
+    // warp-cooperative copies of the runs of the warp's 32 slots: one warp
+    // instruction moves one run type (partner runs, then own-slot runs) of
+    // SPI = 32 / NP consecutive slots, lane l taking 16-byte piece l % NP of
+    // slot l / NP's run -- a few whole runs per instruction (contiguous
+    // pieces, ~2 lines each) instead of 32 pieces of 32 different runs.
+    // Lane l's (slot offset, piece) is fixed, so an instruction costs one
+    // 64-bit pointer shuffle and compile-time shared-memory offsets (the
+    // former piece-by-piece mapping spent ~25 instructions per copy on its
+    // divisions and three shuffles: 31 % of the kernel's instructions).
     constexpr int NP = SM::SPP / 4;           // 16-byte pieces per run
+    constexpr int SPI = 32 / NP;              // slots per warp instruction
+    static_assert(SPI >= 1, "a run must fit one warp instruction");
+    constexpr int NINS = (32 + SPI - 1) / SPI;
     const int lane = gt & 31;
     const int wbase = gt - lane;
+    const int so = lane / NP, qo = 4 * (lane - so * NP);
+    const bool act = so < SPI;
+    int32_t* const dst0 = s_E + (wbase + so) * RS + qo;
 #pragma unroll
     for (int i = 0; i < NJ; ++i) {
+      const int32_t* pa = eprows(gs[i]) + colA[i];
+      const int32_t* pb = eprows(gs[i]) + colB[i];
 #pragma unroll
-      for (int ins = 0; ins < 2 * NP; ++ins) {
-        const int P = ins * 32 + lane;
-        const int r = P / NP;                 // run of the warp: 2 per slot
-        const int q = P - r * NP;
-        const int sl = r >> 1;
-        const int32_t gr = __shfl_sync(0xffffffffu, gs[i], sl);
-        const int32_t cA = __shfl_sync(0xffffffffu, colA[i], sl);
-        const int32_t cB = __shfl_sync(0xffffffffu, colB[i], sl);
-        const int32_t js = wbase + sl + i * GT;
-        if (js < Lc)
-          cp_async16(s_E + js * RS + ((r & 1) ? SM::SP : 0) + 4 * q, eprows(gr) + ((r & 1) ? cB : cA) + 4 * q);
+      for (int run = 0; run < 2; ++run) {
+#pragma unroll
+        for (int ins = 0; ins < NINS; ++ins) {
+          const int sl = ins * SPI + so;      // the slot (of the warp's 32) this lane copies for
+          const int32_t* src = (const int32_t*)__shfl_sync(0xffffffffu, (unsigned long long)(run ? pb : pa), sl & 31);
+          if (act && sl < 32 && wbase + sl + i * GT < Lc)
+            cp_async16(dst0 + (ins * SPI + i * GT) * RS + (run ? SM::SP : 0), src + qo);
+        }
       }
     }
   }
   if (spec && gt < 6) s_E[SM::MOFF + gt] = 0;
+  const unsigned long long t_iss = tprof ? gtimer() : 0;
   cp_async_wait_all();
   group_sync(bar_id, GT);
   unsigned long long t0 = tprof ? gtimer() : 0;
+  if (tprof) { tprof[1] += t_iss - t_in; tprof[2] += t0 - t_iss; }
   // ---- Tp classes on the extended range: thread gt takes pair k = a + gt,
   // valid while t <= tmax (the trapezoid); its local slots are linear in t ----
   int mysw = 0;
@@ -511,7 +530,9 @@ k_ls_trap(const TrapParams p) {
   // PM_TRAP_PROF = 1: CTA 0, 2: the last CTA, 3: the middle one
   const unsigned pblk = p.prof == 2 ? nblk - 1 : (p.prof == 3 ? nblk / 2 : 0);
   const bool prof = p.prof && blockIdx.x == pblk && threadIdx.x == 0 && p.max_log >= 200;
-  unsigned long long t_ld = 0, t_st = 0, t_bar = 0, t_pub = 0, n_ph = 0, tq = prof ? gtimer() : 0;
+  unsigned long long t_ld = 0, t_bar = 0, t_pub = 0, n_ph = 0, tq = prof ? gtimer() : 0;
+  unsigned long long t_stv[3] = {0, 0, 0}, t_fw = 0;   // steps, issue, copy wait; neighbour-flag wait
+  unsigned long long& t_st = t_stv[0];
   const unsigned long long t_start0 = tq;
   const int npass = (p.nchunks + ngrp_tot - 1) / ngrp_tot;
   uint32_t nph_cl = 0;   // cluster mode: phases completed (mbarrier parity)
@@ -539,7 +560,7 @@ k_ls_trap(const TrapParams p) {
             const int2* rr = rep + cur * S;
             mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, er, aligned, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) { const int2 v = rr[x]; g = v.x; d = v.y; el = -1; },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, epr, spec, p.coal);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? t_stv : nullptr, epr, spec, p.coal);
           } else {
             const int bi = p.nbsync ? (int)(qph % 3u) : cur;
             const int4* __restrict__ sc = bi == 0 ? p.sbuf[0] : (bi == 1 ? p.sbuf[1] : p.sbuf[2]);
@@ -547,6 +568,7 @@ k_ls_trap(const TrapParams p) {
               // the neighbour chunks' slots of phase qph - 1 (W >= 2T: every
               // reader of this buffer's previous generation is within two
               // chunks, and those finished it before our neighbours did theirs)
+              const unsigned long long tw0 = prof ? gtimer() : 0;
               if (gt == 0) {
 #pragma unroll
                 for (int dch = -1; dch <= 1; dch += 2) {
@@ -559,12 +581,13 @@ k_ls_trap(const TrapParams p) {
                 }
               }
               group_sync(1 + grp, GT);
+              if (prof) t_fw += gtimer() - tw0;
             }
             mysw += trap_chunk<PPL, T, EP>(C, k0, k1, c0, u0, er, aligned, S,
                                        [&](int32_t x, int32_t& g, int32_t& d, int32_t& el) {
                                          const int4 v = __ldcg(sc + x); g = v.x; d = v.y; el = v.z;
                                        },
-                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? &t_st : nullptr, epr, spec, p.coal);
+                                       s_st, s_g, s_E, gt, 1 + grp, vec, prof ? t_stv : nullptr, epr, spec, p.coal);
           }
           if (prof) { const unsigned long long t = gtimer(); t_ld += t - tq; tq = t; }
           // ---- publish the slots of the owned pairs (class c0 + Tp - 1) ----
@@ -667,6 +690,7 @@ k_ls_trap(const TrapParams p) {
     p.per_round[192] = (int64_t)(t_ld - t_st); p.per_round[193] = (int64_t)t_st;
     p.per_round[194] = (int64_t)t_bar; p.per_round[195] = (int64_t)n_ph;
     p.per_round[196] = (int64_t)t_pub;
+    p.per_round[198] = (int64_t)t_fw; p.per_round[199] = (int64_t)t_stv[1]; p.per_round[200] = (int64_t)t_stv[2];
   }
   if (CLU) {
     // every CTA writes the slots of its owned pairs in the last class

@@ -31,10 +31,11 @@ for cfg in cfgs:
         st = pm.lib().pm_local_search_ex(E.data_ptr(), E.stride(0), S, perm.data_ptr(), int(os.environ.get("PM_MAX_ROUNDS", "0")), pm.METHODS["trap"],
                                          ctypes.byref(r), ctypes.byref(sw), per.ctypes.data, 256, None)
     ld, stp, bar, nph, pub, t0 = per[192:198]
+    fw, iss, cpw = per[198:201]
     nph = max(int(nph), 1)
     ends = [int(x) for x in per[224:256] if x > 0]
     rt = np.diff([int(t0)] + ends) / 1e3
     print(f"cfg{cfg} S={S} st={st} rounds={r.value} phases={nph} per phase: stage {ld/nph:.0f} ns, "
-          f"steps {stp/nph:.0f} ns, publish {pub/nph:.0f} ns, publish+barrier {bar/nph:.0f} ns; total "
+          f"[flag wait {fw/nph:.0f}, state+issue {iss/nph:.0f}, copy wait {cpw/nph:.0f}] steps {stp/nph:.0f} ns, publish {pub/nph:.0f} ns, publish+barrier {bar/nph:.0f} ns; total "
           f"{(ld+stp+bar)/1e6:.3f} ms; TRAP rounds (us) {np.round(rt, 1).tolist()} swaps {per[:len(rt)].tolist()}",
           flush=True)
