@@ -105,21 +105,25 @@ struct TrapSmem {
 };
 
 
-// Speculative class steps pay only once nearly every chunk's phase is quiet:
-// a pass (every remaining class tested, the first firing class applied) costs
-// a few chain steps, and a phase needs 1 + (firing classes) passes, so busy
-// chunks get slower while quiet ones get faster -- and in the chain of
-// neighbour-synchronised chunks the slow ones pace everybody (measured,
-// DESIGN.md).  So they are used from the second round on, when the previous
-// round's swaps predict f = swaps * X * T / (classes * pairs) < 3/4 firing
-// classes per chunk and phase (the previous round's count over-estimates
-// this round's).  mode: trap_spec (0 never, 1 this rule, 2 always).  Results
-// are identical either way.
+// Speculative class steps pay only once most chunk-phases are quiet: a pass
+// (every remaining class tested, the first firing class applied) costs a few
+// chain steps, and a phase needs 1 + (firing classes) passes, so busy chunks
+// get slower while quiet ones get faster -- and in the chain of
+// neighbour-synchronised chunks the slow ones pace everybody.  The firing
+// classes per chunk and phase of this round are predicted from the previous
+// round's swaps, which fall ~3x per round from round 1 on: f = (prev / 3) *
+// X * T / (classes * pairs).  Crossovers measured per mode (round 2,
+// DESIGN.md): grid 192 x 48 (E in HBM) dense wins at f = 0.32 and loses at
+// 0.12 -> threshold 0.2; grid 128 x 32 spec wins at f = 0.39 -> 0.5; cluster
+// mode (DSMEM hand-off, configs 1-2) spec wins up to f ~ 1 -> 1.2.  mode:
+// trap_spec (0 never, 1 this rule, 2 always).  Results are identical either
+// way.
 __device__ __forceinline__ bool spec_round(int32_t mode, int64_t prev_rs, int32_t X, int32_t T, int32_t ncls,
-                                           int32_t npairs) {
+                                           int32_t npairs, bool clu) {
   if (mode == 2) return true;
   if (mode != 1 || prev_rs < 0) return false;
-  return prev_rs * (int64_t)X * T * 4 < (int64_t)ncls * npairs * 3;
+  const int64_t thr10 = clu ? 12 : (T >= 48 ? 2 : 5);   // threshold x 10
+  return prev_rs * (int64_t)X * T * 10 < thr10 * 3 * (int64_t)ncls * npairs;
 }
 
 __device__ __forceinline__ int32_t wrap_m(int32_t x, int32_t m) {
@@ -539,7 +543,7 @@ k_ls_trap(const TrapParams p) {
   uint32_t qph = 0;      // grid mode: phases completed
   int64_t prev_rs = -1;   // swaps of the previous round (-1: none yet)
   for (;;) {
-    const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1);
+    const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1, CLU);
     if (!CLU && blockIdx.x == 0 && threadIdx.x == 0) p.rsw[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
@@ -1100,7 +1104,7 @@ k_ls_trap_mr(const TrapMultiParams p) {
   int status = PM_OK;
   int64_t prev_rs = -1;
   while (ok) {
-    const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1);
+    const bool spec = spec_round(p.spec, prev_rs, X, T, ncls, K + 1, false);
     if (leader) me.rtot[(rounds + 1) % 3] = 0ull;
     for (int32_t c0 = 0; c0 < ncls && ok; c0 += T) {
       const int32_t Tp = min(T, ncls - c0);
