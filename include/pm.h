@@ -167,6 +167,24 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
                                   int32_t max_rounds, int32_t method, int64_t* d_result,
                                   pm_stream_t stream);
 
+/* pm_local_search_async with the sigma-permuted copy of E in a CALLER-OWNED
+ * buffer.  Method TRAP stages its per-tile E runs from
+ * Ep[t][q] = E[t][2q mod m] (q < m + 48 cyclic, m = S-1),
+ * which pm_local_search_async builds in library scratch for every call: at
+ * S = 65536 that is 16 GiB mapped and released per call (~100 ms).  Here the
+ * copy is built into d_Ep instead, so a caller that searches repeatedly
+ * allocates it once.
+ *   pm_sigma_copy_bytes : bytes d_Ep must hold for S (0 for S < 2).
+ *   d_Ep      : device buffer of at least pm_sigma_copy_bytes(S) bytes,
+ *               16-byte aligned, owned by the caller; overwritten (any other
+ *               method leaves it untouched).
+ * Results are identical to pm_local_search_async (Alg. 2).
+ * PM_ERR_INVALID for a NULL or too small d_Ep, else as pm_local_search_async. */
+size_t pm_sigma_copy_bytes(int32_t S);
+pm_status_t pm_local_search_ep_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                     int32_t max_rounds, int32_t method, int32_t* d_Ep, size_t ep_bytes,
+                                     int64_t* d_result, pm_stream_t stream);
+
 /* Multi-GPU Algorithm 2 (method PM_LS_TRAP split across ranks,
  * one rank per GPU of one NVLink box).  The colour classes are global
  * perfect matchings, so the search does not shard into independent parts;

@@ -209,7 +209,7 @@ pm_status_t ls_method_supported(int32_t S, int32_t method) {
 
 pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                              int32_t method, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
-                             cudaStream_t st, int32_t* used_method) {
+                             cudaStream_t st, int32_t* used_method, int32_t* ep_buf, size_t ep_bytes) {
   if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
   if (used_method) *used_method = method;
   {
@@ -222,18 +222,26 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   // first (full) scan streams its rows instead of gathering from E
   ScopedScratch ep(st);
   int64_t ldp = 0;
+  const int32_t* Ep_use = nullptr;
   if (method == PM_LS_TRAP) {
     PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
-    int32_t* Ep = nullptr;
-    const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
-    ep.p = Ep;
-    if (se != PM_OK) return se;
+    if (ep_buf && ep_bytes >= trap_ep_bytes(S)) {   // the caller's buffer (pm_local_search_ep_async)
+      const pm_status_t se = trap_build_ep_into(E, ldE, S, st, ep_buf, &ldp);
+      if (se != PM_OK) return se;
+      Ep_use = ep_buf;
+    } else {
+      int32_t* Ep = nullptr;
+      const pm_status_t se = trap_build_ep(E, ldE, S, st, &Ep, &ldp);
+      ep.p = Ep;
+      if (se != PM_OK) return se;
+      Ep_use = Ep;
+    }
   }
   SparseRun sr;
   ScopedScratch sps(st);
   if (sparse_T > 0) {
     const pm_status_t s = sparse_prepare(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, &sr, 0,
-                                         ep.as<int32_t>(), ldp);
+                                         Ep_use, ldp);
     if (s != PM_OK) return s;
     sps.p = sr.scratch;   // freed here on an error path; sparse_launch frees it otherwise
   }
@@ -244,7 +252,7 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
       break;
     case PM_LS_TRAP:
       s = run_trap(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T,
-                   ep.as<int32_t>(), ldp);
+                   Ep_use, ldp);
       break;
     case PM_LS_WINDOW:
       s = run_window(E, ldE, S, perm, max_rounds, dev_out, dev_per_round, max_log, st, sr.pending, sparse_T);

@@ -829,6 +829,16 @@ static size_t device_total_mem() {
   return t;
 }
 
+int64_t trap_ep_ld(int32_t S) { return ((int64_t)S - 1 + 48 + 31) / 32 * 32; }
+size_t trap_ep_bytes(int32_t S) { return S < 2 ? 0 : sizeof(int32_t) * (size_t)S * (size_t)trap_ep_ld(S); }
+
+pm_status_t trap_build_ep_into(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t* Ep,
+                               int64_t* ldp) {
+  *ldp = trap_ep_ld(S);
+  PM_CUDA_TRY(launch_permute_cols(E, ldE, Ep, *ldp, S, S - 1, 48, st));
+  return PM_OK;
+}
+
 pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
                           int64_t* ldp) {
   *Ep = nullptr;
@@ -836,7 +846,7 @@ pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t
   const int32_t ep_mode = knob("trap_ep", 1);
   if (ep_mode == 0) return PM_OK;
   const int32_t m = S - 1, ext = 48;
-  const int64_t l = ((int64_t)m + ext + 31) / 32 * 32;
+  const int64_t l = trap_ep_ld(S);
   const size_t bytes = sizeof(int32_t) * (size_t)S * (size_t)l;
   if (ep_mode == 1 && bytes > device_total_mem() / 8) return PM_OK;
   *ldp = l;

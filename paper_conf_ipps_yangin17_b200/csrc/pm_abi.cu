@@ -294,6 +294,24 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
                           nullptr, 0, st, &used);
 }
 
+size_t pm_sigma_copy_bytes(int32_t S) { return trap_ep_bytes(S); }
+
+pm_status_t pm_local_search_ep_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                     int32_t max_rounds, int32_t method, int32_t* d_Ep, size_t ep_bytes,
+                                     int64_t* d_result, pm_stream_t stream) {
+  if (!d_result || !d_Ep || ep_bytes < trap_ep_bytes(S) || !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method))
+    return PM_ERR_INVALID;
+  {
+    const pm_status_t v = ls_method_supported(S, method);
+    if (v != PM_OK) return v;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
+  int32_t used = method;
+  return run_local_search(d_E, ld_E, S, d_perm, max_rounds, method, reinterpret_cast<LsResult*>(d_result),
+                          nullptr, 0, st, &used, d_Ep, ep_bytes);
+}
+
 size_t pm_trap_workspace_bytes(int32_t S) { return (S < 2) ? 0 : trap_ws_bytes(S); }
 
 pm_status_t pm_trap_workspace_reset(void* d_ws, int32_t S, pm_stream_t stream) {

@@ -124,7 +124,7 @@ cudaError_t launch_iota(int32_t* perm, int32_t S, cudaStream_t st);
 pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm,
                              int32_t max_rounds, int32_t method, LsResult* dev_out,
                              int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                             int32_t* used_method);
+                             int32_t* used_method, int32_t* ep_buf = nullptr, size_t ep_bytes = 0);
 int32_t ls_class_launches_per_round(int32_t S);
 int32_t ls_window_max_S();
 // Ep[t][pos] = E[t][2 pos mod m], pos in [0, m + ext) (sigma-permuted rows, k_window.cu)
@@ -218,6 +218,11 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
 // TRAP stages from while E <= 2 GiB (trap_ep), or NULL: allocated from the
 // scratch pool on st; the caller frees it.
 pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep, int64_t* ldp);
+// Its leading dimension and size (S rows); built into a caller-owned buffer by
+// trap_build_ep_into (pm_local_search_ep_async).
+int64_t trap_ep_ld(int32_t S);
+size_t trap_ep_bytes(int32_t S);
+pm_status_t trap_build_ep_into(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t* Ep, int64_t* ldp);
 
 // Multi-rank TRAP (k_trap.cu).
 struct TrapRank;

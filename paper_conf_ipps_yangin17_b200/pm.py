@@ -39,6 +39,8 @@ _SIGS = [
     ("pm_local_search", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _P, _P, _P]),
     ("pm_local_search_ex", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P, _P, _I32, _P]),
     ("pm_local_search_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P]),
+    ("pm_sigma_copy_bytes", ctypes.c_size_t, [_I32]),
+    ("pm_local_search_ep_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, ctypes.c_size_t, _P, _P]),
     ("pm_ls_auto_method", _I32, [_I32]),
     ("pm_init_identity", ctypes.c_int, [_P, _I32, _P]),
     ("pm_cost", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P]),
@@ -219,6 +221,20 @@ def local_search_async(E, perm, result, max_rounds: int = 0, method: str = "auto
     _check(lib().pm_local_search_async(E.data_ptr(), E.stride(0), E.shape[0], perm.data_ptr(), max_rounds,
                                        METHODS[method], result.data_ptr(), _stream(stream)),
            "pm_local_search_async")
+
+
+def sigma_copy_bytes(S: int) -> int:
+    """pm_sigma_copy_bytes: size of the caller-owned sigma-permuted copy for S."""
+    return int(lib().pm_sigma_copy_bytes(S))
+
+
+def local_search_ep_async(E, perm, result, Ep, max_rounds: int = 0, method: str = "auto", stream=None):
+    """pm_local_search_ep_async: as local_search_async, with TRAP's sigma-permuted
+    copy of E built into the caller's buffer Ep (CUDA, >= sigma_copy_bytes(S) bytes)."""
+    _check(lib().pm_local_search_ep_async(E.data_ptr(), E.stride(0), E.shape[0], perm.data_ptr(), max_rounds,
+                                          METHODS[method], Ep.data_ptr(), Ep.numel() * Ep.element_size(),
+                                          result.data_ptr(), _stream(stream)),
+           "pm_local_search_ep_async")
 
 
 def local_search_multi_emulated(E, world: int, perm=None, max_rounds: int = 0, stream=None):

@@ -844,3 +844,43 @@ def test_scratch_pool_trim():
     pm.scratch_trim()
     assert pm.scratch_reserved_bytes() == 0
     _check_ls(oracle_E("smooth", 512, 16), "trap")           # the pool refills on demand
+
+
+# ---- pm_local_search_ep_async: TRAP's sigma-permuted copy in a caller-owned
+# buffer (allocated once, reused across searches) -- same result as the oracle
+@pytest.mark.parametrize("N,M,fam,method", [(128, 8, "smooth", "auto"), (512, 16, "ties", "trap"),
+                                            (512, 16, "smooth", "auto"), (240, 8, "noise", "window"),
+                                            (200, 10, "smooth", "class")])
+def test_local_search_caller_owned_sigma_copy(N, M, fam, method):
+    E_np = oracle_E(fam, N, M)
+    S = E_np.shape[0]
+    if not _supported(method, S):
+        pytest.skip(f"{method} does not take S = {S}")
+    ref = oracle.local_search(E_np)
+    E = dev(E_np)
+    nbytes = pm.sigma_copy_bytes(S)
+    assert nbytes == 4 * S * (((S - 1 + 48 + 31) // 32) * 32)
+    Ep = torch.full((nbytes // 4,), -7, dtype=torch.int32, device=DEV)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    for _ in range(2):   # the same buffer twice
+        perm = torch.arange(S, dtype=torch.int32, device=DEV)
+        pm.local_search_ep_async(E, perm, res, Ep, method=method)
+        torch.cuda.synchronize()
+        assert res.cpu().tolist() == [ref[4], ref[1], ref[2]]
+        assert (perm.cpu().numpy() == ref[0]).all()
+    if method in ("auto", "trap"):   # the copy itself: Ep[t][q] = E[t][2q mod m], q < m + 48 cyclic
+        m, ld = S - 1, nbytes // 4 // S
+        q = np.arange(m + 48)
+        assert (Ep.view(S, ld)[:, : m + 48].cpu().numpy() == E_np[:, (2 * q) % m]).all()
+
+
+def test_local_search_caller_owned_sigma_copy_too_small_rejected():
+    E_np = oracle_E("smooth", 128, 8)
+    S = E_np.shape[0]
+    E = dev(E_np)
+    Ep = torch.empty(pm.sigma_copy_bytes(S) // 4 - 4, dtype=torch.int32, device=DEV)
+    perm = torch.arange(S, dtype=torch.int32, device=DEV)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    with pytest.raises(pm.PMError) as e:
+        pm.local_search_ep_async(E, perm, res, Ep, method="trap")
+    assert e.value.status == pm.PM_ERR_INVALID

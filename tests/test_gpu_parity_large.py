@@ -97,6 +97,18 @@ def test_cfg4_local_search(cfg4, method):
     assert pm.cost(E_gpu, got[0]) == oracle.cost(E_or, ref[0])
 
 
+def test_cfg4_caller_owned_sigma_copy(cfg4):
+    # pm_local_search_ep_async: the 1 GiB sigma-permuted copy in a torch buffer
+    I, T, E_or, E_gpu, ref = cfg4
+    S = E_gpu.shape[0]
+    Ep = torch.empty(pm.sigma_copy_bytes(S) // 4, dtype=torch.int32, device=DEV)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    perm = torch.arange(S, dtype=torch.int32, device=DEV)
+    pm.local_search_ep_async(E_gpu, perm, res, Ep)
+    st, rounds, swaps = res.cpu().tolist()
+    _assert_search((perm, rounds, swaps, None, st), ref, E_or, "config 4 auto, caller-owned sigma copy")
+
+
 def test_cfg4_trap_every_round(cfg4):
     # the sparse hand-over off: every round (incl. the quiet ones) on TRAP
     I, T, E_or, E_gpu, ref = cfg4

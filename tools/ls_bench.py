@@ -9,6 +9,8 @@ import torch  # noqa: E402
 from paper_conf_ipps_yangin17_b200 import pm, synth  # noqa: E402
 sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 import _devknobs  # noqa: E402
+if os.environ.get("PM_LIB"):   # a development build of the library
+    pm.LIB_PATH = os.environ["PM_LIB"]
 _devknobs.apply(pm)
 
 cfgs = [int(c) for c in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["1", "2", "3"])]
