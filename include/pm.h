@@ -371,7 +371,7 @@ int64_t pm_launch_count(void);
  * environment).  Results stay bit-exact under every override -- only speed
  * and the set of supported S change (an override that a launch cannot honour
  * returns PM_ERR_UNSUPPORTED from the search).
- *   name  : one of "trap_variant" (chunk geometry 0..5), "trap_W" (owned
+ *   name  : one of "trap_variant" (chunk geometry 0..7), "trap_W" (owned
  *           pairs per chunk), "trap_cluster" (0 grid, 1 cluster), "trap_nbsync",
  *           "trap_cpc", "trap_ep" (sigma-permuted staging: 0 off, 1 auto,
  *           2 always), "trap_vec", "trap_spec" (speculative class steps: 0 off, 1 quiet rounds,

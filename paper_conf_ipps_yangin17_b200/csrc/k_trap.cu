@@ -113,8 +113,8 @@ struct TrapSmem {
 // classes per chunk and phase of this round are predicted from the previous
 // round's swaps, which fall ~3x per round from round 1 on: f = (prev / 3) *
 // X * T / (classes * pairs).  Crossovers measured per mode (round 2,
-// DESIGN.md): grid 192 x 48 (E in HBM) dense wins at f = 0.32 and loses at
-// 0.12 -> threshold 0.2; grid 128 x 32 spec wins at f = 0.39 -> 0.5; cluster
+// DESIGN.md): grid 192 x 48 (E in HBM; also 224 x 44) dense wins at f = 0.32
+// and loses at 0.12 -> threshold 0.2; grid 128 x 32 spec wins at f = 0.39 -> 0.5; cluster
 // mode (DSMEM hand-off, configs 1-2) spec wins up to f ~ 1 -> 1.2.  mode:
 // trap_spec (0 never, 1 this rule, 2 always).  Results are identical either
 // way.
@@ -122,7 +122,7 @@ __device__ __forceinline__ bool spec_round(int32_t mode, int64_t prev_rs, int32_
                                            int32_t npairs, bool clu) {
   if (mode == 2) return true;
   if (mode != 1 || prev_rs < 0) return false;
-  const int64_t thr10 = clu ? 12 : (T >= 48 ? 2 : 5);   // threshold x 10
+  const int64_t thr10 = clu ? 12 : (X >= 192 ? 2 : 5);   // threshold x 10
   return prev_rs * (int64_t)X * T * 10 < thr10 * 3 * (int64_t)ncls * npairs;
 }
 
@@ -921,6 +921,7 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
     case 4: return launch_trap<4, 8>(hp, st);
     case 5: return launch_trap<4, 32>(hp, st);
     case 6: return launch_trap<6, 48>(hp, st);
+    case 7: return launch_trap<7, 44>(hp, st);
     default:
       // measured (whole search, configs 1/2/3/4): 128-pair ranges
       // x 32 classes 0.338/1.049/6.14/36.6 ms, 64 x 16 0.353/1.172/7.73/54.9,
@@ -929,7 +930,20 @@ pm_status_t run_trap(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, in
       // from E's own rows (E > 2 GiB, config 5) 64 x 16 (round 1: 1.21 vs
       // 1.32 s for 128 x 32)
       if (!hp.Ep) return launch_trap<2, 16>(hp, st);
-      if ((int64_t)S * ldE * 4 > (96ll << 20)) return launch_trap<6, 48>(hp, st);
+      if ((int64_t)S * ldE * 4 > (96ll << 20)) {
+        // 192 x 48 (96 owned pairs) unless its chunks need more passes per
+        // phase over the SMs than 224 x 44 (136 owned pairs, 222 KB of
+        // staging): config 5 has 342 chunks = 3 passes on 148 SMs, 241 = 2
+        // passes (measured: TRAP round 34 -> ~24 ms); config 4
+        // (86 chunks) keeps 192 x 48
+        int dev = 0, nsm = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        const int64_t np = Classes(S).npairs;
+        const int64_t pass48 = ((np + 95) / 96 + nsm - 1) / nsm, pass44 = ((np + 135) / 136 + nsm - 1) / nsm;
+        if (pass44 < pass48) return launch_trap<7, 44>(hp, st);
+        return launch_trap<6, 48>(hp, st);
+      }
       return launch_trap<4, 32>(hp, st);
   }
 }

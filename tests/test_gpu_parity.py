@@ -553,7 +553,7 @@ def _check_trap(E_np, cluster_forced=False):
 # ---- PM_LS_TRAP: every round on the temporal-blocked kernel (sparse hand-over
 # off), every compiled (pairs-per-lane, T) variant, chunk widths that do not
 # divide S/2, grid-barrier and cluster (DSMEM) modes.
-@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4, 5, 6])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4, 5, 6, 7])
 @pytest.mark.parametrize("N,M,fam,W", [(128, 8, "smooth", 0), (512, 16, "smooth", 0), (512, 16, "ties", 7),
                                        (240, 8, "noise", 0), (336, 8, "smooth", 21), (128, 8, "transposition", 19)])
 @pytest.mark.parametrize("mode", ["0", "1"])
@@ -566,7 +566,7 @@ def test_trap_every_round(variant, N, M, fam, W, mode):
 
 
 @pytest.mark.parametrize("spec", [0, 1, 2])
-@pytest.mark.parametrize("variant", [0, 1, 3, 5, 6])
+@pytest.mark.parametrize("variant", [0, 1, 3, 5, 6, 7])
 @pytest.mark.parametrize("N,M,fam", [(512, 16, "smooth"), (512, 16, "ties"), (336, 8, "smooth"), (1024, 16, "smooth")])
 @pytest.mark.parametrize("mode", ["0", "1"])
 def test_trap_speculative_steps(spec, variant, N, M, fam, mode):
