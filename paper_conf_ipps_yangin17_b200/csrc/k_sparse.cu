@@ -70,53 +70,52 @@ __global__ void k_sp_begin(SpParams* p, cudaGraphConditionalHandle h) {
 // partner in class c is (2c+1-y) mod m, whose sigma-position is
 // (c + (m+1)/2 - sigma(y)) mod m: consecutive classes read consecutive
 // entries of row r[y].  So with w_y(c) = E[r[y]][partner_c(y)] - d[y], the
-// pair (u, v) of class c fires iff w_u(c) + w_v(c) < 0 (line 5), and a tile
-// of kScanU slots x kScanB classes needs the streams of its slots and of the
-// kScanU + 2 kScanB - 2 partner slots over those classes -- coalesced rows
-// instead of two scattered gathers per pair.  The fixed point u0 of each
-// class and slot S-1 (even S) are tested separately.
-constexpr int kScanU = 256, kScanB = 32, kScanVB = kScanU + 2 * kScanB;
-constexpr size_t kScanSmem = sizeof(int32_t) * (size_t)(kScanU + kScanVB) * kScanB;
+// pair (u, v) of class c fires iff w_u(c) + w_v(c) < 0 (line 5).  Tiles are
+// taken in pair-index space: pairs k0 .. k0+kScanP-1 over classes
+// c0 .. c0+kScanB-1 hold first slots u0(c0)+t+k and second slots
+// u0(c0)+t-k -- two contiguous ranges of kScanP+kScanB-1 slots -- so a tile
+// streams each of those slots' 128-byte runs once and tests every pair once
+// (a slot-block tiling tests each pair from both of its slots and streams
+// every run twice: config 4 first scan 1.07 ms).  Pair 0 (u0, S-1) of even S
+// is tested separately.
+constexpr int kScanP = 256, kScanB = 32;
+constexpr int kScanR = (kScanP + kScanB - 1 + 31) / 32 * 32;   // rows per side (287 -> 288)
+constexpr size_t kScanSmem = sizeof(int32_t) * (size_t)(2 * kScanR) * kScanB;
 
 __device__ __forceinline__ void scan_full_ep(const SpParams* __restrict__ p, int32_t stamp, int32_t* sm) {
   const Classes cl(p->S);
   const int32_t m = cl.m, H = cl.half, S = p->S;
+  const int32_t KR = (m - 1) / 2;        // regular pairs k = 1 .. KR
   const int32_t* __restrict__ r = p->r;
   const int32_t* __restrict__ d = p->d;
   const int32_t* __restrict__ Ep = p->Ep;
   const int64_t ldp = p->ldp;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
-  int32_t* wA = sm;                      // [kScanU][kScanB]
-  int32_t* wB = sm + kScanU * kScanB;    // [kScanVB][kScanB]
-  const int32_t nU = (m + kScanU - 1) / kScanU, nC = (m + kScanB - 1) / kScanB;
-  for (int32_t tile = blockIdx.x; tile < nU * nC; tile += gridDim.x) {
-    const int32_t x0 = (tile % nU) * kScanU, c0 = (tile / nU) * kScanB;
-    int32_t vbase = (int32_t)(((int64_t)2 * c0 + 1 - x0 - (kScanU - 1)) % m);
-    vbase = vbase < 0 ? vbase + m : vbase;
+  int32_t* wA = sm;                      // [kScanR][kScanB]: first slots
+  int32_t* wB = sm + kScanR * kScanB;    // [kScanR][kScanB]: second slots
+  const int32_t nP = (KR + kScanP - 1) / kScanP, nC = (m + kScanB - 1) / kScanB;
+  for (int32_t tile = blockIdx.x; tile < nP * nC; tile += gridDim.x) {
+    const int32_t k0 = 1 + (tile % nP) * kScanP, c0 = (tile / nP) * kScanB;
+    // row j of side A is slot u0(c0) + k0 + j, of side B slot u0(c0) - k0 - (kScanP-1) + j (mod m)
+    int32_t baseA = (int32_t)(((int64_t)c0 + H + k0) % m);
+    int32_t baseB = (int32_t)(((int64_t)c0 + H - k0 - (kScanP - 1)) % m);
+    baseB = baseB < 0 ? baseB + m : baseB;
     const int32_t c = c0 + lane;
     // rows in groups of 32 per warp: lane l fetches row l's tile, d and start
     // position (coalesced), then the warp streams the 32 rows' class runs
     // (one 128-byte load each, all in flight together)
-    constexpr int NG = (kScanU + kScanVB) / 32;
+    constexpr int NG = 2 * kScanR / 32;
     for (int32_t grp = warp; grp < NG; grp += nwarp) {
-      const int32_t row = grp * 32 + lane;
-      int32_t y;
-      bool ok = true;
-      if (row < kScanU) {
-        y = x0 + row;
-        ok = y < m;
-      } else {
-        y = (vbase + (row - kScanU)) % m;   // (m may be below kScanVB: rows then repeat)
-      }
-      int32_t t = 0, dy = 0, q = 0;
-      if (ok) {
-        t = __ldg(r + y);
-        dy = __ldg(d + y);
-        // sigma-position of class c0's partner: c0 + H - sigma(y) mod m, where
-        // sigma(y) = y H mod m is y/2 or (y+m)/2 (m odd) -- no 64-bit remainder
-        q = c0 + H - ((y & 1) ? (y + m) >> 1 : y >> 1);
-        q = q < 0 ? q + m : (q >= m ? q - m : q);
-      }
+      const bool sideA = grp < kScanR / 32;
+      const int32_t row = (sideA ? grp : grp - kScanR / 32) * 32 + lane;
+      int32_t y = (sideA ? baseA : baseB) + row;   // < 3m
+      y = y >= m ? y - m : y;
+      y = y >= m ? y - m : y;
+      const int32_t t = __ldg(r + y), dy = __ldg(d + y);
+      // sigma-position of class c0's partner: c0 + H - sigma(y) mod m, where
+      // sigma(y) = y H mod m is y/2 or (y+m)/2 (m odd) -- no 64-bit remainder
+      int32_t q = c0 + H - ((y & 1) ? (y + m) >> 1 : y >> 1);
+      q = q < 0 ? q + m : (q >= m ? q - m : q);
       int32_t val[32];
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
@@ -124,27 +123,20 @@ __device__ __forceinline__ void scan_full_ep(const SpParams* __restrict__ p, int
         const int32_t qi = __shfl_sync(0xffffffffu, q, i);
         val[i] = __ldg(Ep + (int64_t)ti * ldp + qi + lane);   // qi + lane < m + 32 <= ldp (cyclic copy)
       }
+      int32_t* dst = (sideA ? wA : wB) + (row - lane) * kScanB;
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
         const int32_t di = __shfl_sync(0xffffffffu, dy, i);
-        const int32_t oi = __shfl_sync(0xffffffffu, ok ? 1 : 0, i);
-        const int32_t ri = grp * 32 + i;
-        int32_t* dst = ri < kScanU ? wA + ri * kScanB : wB + (ri - kScanU) * kScanB;
-        dst[lane] = (oi && c < m) ? val[i] - di : 0;
+        dst[i * kScanB + lane] = val[i] - di;
       }
     }
     __syncthreads();
     if (c < m) {
-      int32_t u0 = c + H;
-      u0 = u0 >= m ? u0 - m : u0;
-      for (int32_t ur = warp; ur < kScanU; ur += nwarp) {
-        const int32_t u = x0 + ur;
-        if (u >= m || u == u0) continue;
-        int32_t v = 2 * c + 1 - u;
-        v = v < 0 ? v + m : (v >= m ? v - m : v);
-        int32_t vr = v - vbase;
-        vr = vr < 0 ? vr + m : vr;
-        if ((int64_t)wA[ur * kScanB + lane] + wB[vr * kScanB + lane] < 0) p->flags[c] = stamp;
+      // pair k = k0 + kk at class c0 + lane: first slot = row lane + kk of A,
+      // second slot = row lane + kScanP-1 - kk of B (conflict-free: bank = lane)
+      for (int32_t kk = warp; kk < kScanP && k0 + kk <= KR; kk += nwarp) {
+        if ((int64_t)wA[(lane + kk) * kScanB + lane] + wB[(lane + kScanP - 1 - kk) * kScanB + lane] < 0)
+          p->flags[c] = stamp;
       }
     }
     __syncthreads();
