@@ -220,7 +220,7 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def rooflines(cfg, S, P, rounds, ls_ms, e_ms, e_rows, sm_max, method_used):
+def rooflines(cfg, S, P, rounds, ls_ms, e_ms, e_rows, sm_max, method_used, sigma_fused=False):
     """Dominant-kernel roofline objects: Alg. 2 against HBM
     with its algorithmic 8 bytes per pair evaluation, the E kernel against
     the VABSDIFF4 ALU peak with P byte-absdiffs per pair."""
@@ -235,10 +235,12 @@ def rooflines(cfg, S, P, rounds, ls_ms, e_ms, e_rows, sm_max, method_used):
                "peak": hbm_peak, "unit": "GB/s", "frac": ls_gbs / hbm_peak,
                "traffic": ncu_traffic("k_ls_trap", cfg) if method_used == "trap" else None,
                "peak_source": hbm_src, "algorithmic_bytes": ls_bytes,
-               "timing": "CUDA events around the pm_local_search_async call on its stream, mean over the timed steps",
+               "timing": "CUDA events around the local-search call on its stream, mean over the timed steps",
                "note": "latency-bound chain of S-1 dependent class steps per round; "
                        "algorithmic bytes = rounds * S(S-1)/2 * 8 (2 int32 E gathers per pair evaluation)"}
-    roof_e = {"kernel": "k_sad (Eq. 1 SAD-GEMM, VABSDIFF4) + k_pack (Step 1)", "bound": "alu",
+    roof_e = {"kernel": "k_sad (Eq. 1 SAD-GEMM, VABSDIFF4) + k_pack (Step 1)"
+                        + (", whose epilogue also writes the sigma-permuted copy of E (1 more int32 store per entry; "
+                           "the search then skips k_permute_cols)" if sigma_fused else ""), "bound": "alu",
               "achieved": e_tops, "peak": alu_peak, "unit": "T byte-absdiff/s", "frac": e_tops / alu_peak,
               "traffic": ncu_traffic("k_sad", cfg),
               "peak_source": f"derived: 148 SM x {ALU_VABSDIFF4_PER_CLK_PER_SM} VABSDIFF4/clk (measured issue "
@@ -270,13 +272,25 @@ def bench_single(args, rank, world, local_rank):
     flush = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
+    # TRAP stages from the sigma-permuted copy of E: write it in the E pass
+    # (pm_error_matrix_sigma) into a buffer allocated once, as
+    # pm_photomosaic_async does internally
+    use_sigma = (pm.ls_auto_method(S) if args.method == "auto" else args.method) == "trap"
+    Ep = torch.empty(pm.sigma_copy_bytes(S) // 4 if use_sigma else 1, dtype=torch.int32, device=dev)
+
     def step(evs=None):
         # the public ABI pieces of pm_photomosaic_async, with events between them
         if evs: evs[0].record(stream)
-        pm.error_matrix(dI, dT, M, out=E)                      # Step 1 + Step 2
+        if use_sigma:
+            pm.error_matrix_sigma(dI, dT, M, E, Ep)            # Step 1 + Step 2 (+ the sigma copy)
+        else:
+            pm.error_matrix(dI, dT, M, out=E)                  # Step 1 + Step 2
         if evs: evs[1].record(stream)
         pm.init_identity(perm)
-        pm.local_search_async(E, perm, res[:3], method=args.method)
+        if use_sigma:
+            pm.local_search_sigma_async(E, perm, res[:3], Ep, method=args.method)
+        else:
+            pm.local_search_async(E, perm, res[:3], method=args.method)
         if evs: evs[2].record(stream)
         pm.cost_async(E, perm, res[3:])
         if evs: evs[3].record(stream)
@@ -339,7 +353,7 @@ def bench_single(args, rank, world, local_rank):
     rounds = out_res[1]
     sm_max = clk.max_mhz or 1965
     used = pm.ls_auto_method(S) if args.method == "auto" else args.method
-    dominant, other = rooflines(args.config, S, P, rounds, mean_ls, mean_e, S, sm_max, used)
+    dominant, other = rooflines(args.config, S, P, rounds, mean_ls, mean_e, S, sm_max, used, use_sigma)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
@@ -354,7 +368,9 @@ def bench_single(args, rank, world, local_rank):
                 "api": "pm_photomosaic_host (pinned host images -> host r)"},
         "gpu_launches": launches,
         "roofline": dominant, "roofline_other": other,
-        "breakdown_ms": {"pack+error_matrix": mean_e, "local_search": mean_ls, "cost": statistics.mean(cost_ms)},
+        "breakdown_ms": {"pack+error_matrix": mean_e, "local_search": mean_ls, "cost": statistics.mean(cost_ms),
+                         "note": ("the E pass also writes TRAP's sigma-permuted copy of E (pm_error_matrix_sigma); "
+                                  "the search runs on it (pm_local_search_sigma_async)") if use_sigma else ""},
         "local_search": {"method": used, "rounds": rounds, "class_steps": rounds * max(S - 1, 1),
                          "ns_per_class_step": mean_ls * 1e6 / (rounds * max(S - 1, 1))},
         "result": {"rounds": rounds, "swaps": out_res[2], "cost": out_res[3]},

@@ -133,6 +133,7 @@ struct SadGeom {
   int64_t rowbytes;        // image: N*C
   int32_t a_tile0;         // image: tile index of local row 0 (row_begin)
   int32_t g, M, R, MC;     // image: tiles per grid row, tile side, pieces per tile row, M*C
+  int32_t e_row0;          // row of Ep that local row 0 goes to (the sigma copy, when written)
 };
 
 template <bool kImage>
@@ -150,7 +151,8 @@ __device__ __forceinline__ const uint8_t* sad_tile_base(const SadGeom& geo, cons
 // 148 SMs with 128 x 128 tiles without split-K).
 template <bool kAtomic, bool kImage, int BN>
 __global__ void __launch_bounds__(sad::kThreads, BN == 128 ? 1 : 2)
-k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE) {
+k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE,
+      int32_t* __restrict__ Ep, int64_t ldp) {
   using namespace sad;
   constexpr int NJ = BN / 16;                          // output columns per thread
   extern __shared__ __align__(16) uint32_t smem[];
@@ -250,6 +252,20 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
       if (col >= S) continue;
       if (kAtomic) atomicAdd(erow + col, (int32_t)acc[i][j]);
       else erow[col] = (int32_t)acc[i][j];
+      // the sigma-permuted copy TRAP stages from (k_trap.cu), written in the
+      // same pass (no separate read + write of E): Ep[row][q] = E[row][2q mod m]
+      // for q < m + 48 cyclic, m = S - 1 odd -> column col lands at
+      // q = sigma(col) = col/2 (even) or (col+m)/2 (odd), and again at q + m
+      // when q < 48
+      if (!kAtomic && Ep) {
+        const int32_t m = S - 1;
+        if (col < m) {
+          const int32_t q = (col & 1) ? (col + m) >> 1 : col >> 1;
+          int32_t* prow = Ep + (int64_t)(geo.e_row0 + row) * ldp;
+          prow[q] = (int32_t)acc[i][j];
+          if (q < 48) prow[q + m] = (int32_t)acc[i][j];
+        }
+      }
     }
   }
 }
@@ -296,7 +312,8 @@ static cudaError_t sad_set_attr() {
 }
 
 static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows, int32_t S, int32_t P,
-                                   int32_t* E, int64_t ldE, cudaStream_t st) {
+                                   int32_t* E, int64_t ldE, cudaStream_t st, int32_t* Ep = nullptr,
+                                   int64_t ldp = 0) {
   using namespace sad;
   if (nrows <= 0 || S <= 0) return cudaSuccess;
   int dev = 0, sms = 148;
@@ -331,32 +348,41 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
   if (plan.bn == 64) {
     dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, (unsigned)split);
     if (split > 1) {
-      if (image) k_sad<true, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE);
-      else k_sad<true, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE);
+      if (image) k_sad<true, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
+      else k_sad<true, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
     } else {
-      if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
-      else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE);
+      if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
+      else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
     }
     note_launch();
     return cudaGetLastError();
   }
   dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
-  if (split > 1) {
-    if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE);
-    else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE);
+  if (split > 1) {   // (split-K accumulates: the sigma copy follows E, launch_sad_sigma)
+    if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
+    else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
   } else {
-    if (image) k_sad<false, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE);
-    else k_sad<false, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE);
+    if (image) k_sad<false, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
+    else k_sad<false, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
   }
   note_launch();
   return cudaGetLastError();
 }
 
 cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
-                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st) {
+                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st, int32_t* Ep, int64_t ldp,
+                       int32_t row0) {
   SadGeom geo = {};
   geo.A = A; geo.B = B; geo.ldt = ldt;
-  return launch_sad_geom(geo, false, nrows, S, P, E, ldE, st);
+  geo.e_row0 = row0;
+  return launch_sad_geom(geo, false, nrows, S, P, E, ldE, st, Ep, ldp);
+}
+
+bool sad_split_plan(int32_t nrows, int32_t S, int32_t P) {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return choose_plan(nrows, S, (P / 4) / sad::BKW, sms).split > 1;
 }
 
 bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C) {
@@ -366,14 +392,16 @@ bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int3
 }
 
 cudaError_t launch_sad_image(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C,
-                             int32_t row_begin, int32_t row_end, int32_t* E, int64_t ldE, cudaStream_t st) {
+                             int32_t row_begin, int32_t row_end, int32_t* E, int64_t ldE, cudaStream_t st,
+                             int32_t* Ep, int64_t ldp) {
   SadGeom geo = {};
   geo.A = I; geo.B = T;
+  geo.e_row0 = row_begin;
   geo.rowbytes = (int64_t)N * C;
   geo.a_tile0 = row_begin;
   geo.g = N / M; geo.M = M; geo.MC = M * C; geo.R = M * C / 16;
   const int32_t S = geo.g * geo.g;
-  return launch_sad_geom(geo, true, row_end - row_begin, S, M * M * C, E, ldE, st);
+  return launch_sad_geom(geo, true, row_end - row_begin, S, M * M * C, E, ldE, st, Ep, ldp);
 }
 
 }  // namespace pm

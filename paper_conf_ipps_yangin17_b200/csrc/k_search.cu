@@ -209,7 +209,8 @@ pm_status_t ls_method_supported(int32_t S, int32_t method) {
 
 pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm, int32_t max_rounds,
                              int32_t method, LsResult* dev_out, int64_t* dev_per_round, int32_t max_log,
-                             cudaStream_t st, int32_t* used_method, int32_t* ep_buf, size_t ep_bytes) {
+                             cudaStream_t st, int32_t* used_method, int32_t* ep_buf, size_t ep_bytes,
+                             bool ep_ready) {
   if (method == PM_LS_AUTO) method = pm_ls_auto_method(S);
   if (used_method) *used_method = method;
   {
@@ -225,9 +226,13 @@ pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* 
   const int32_t* Ep_use = nullptr;
   if (method == PM_LS_TRAP) {
     PM_CUDA_TRY(launch_perm_check(perm, S, dev_out, st));
-    if (ep_buf && ep_bytes >= trap_ep_bytes(S)) {   // the caller's buffer (pm_local_search_ep_async)
-      const pm_status_t se = trap_build_ep_into(E, ldE, S, st, ep_buf, &ldp);
-      if (se != PM_OK) return se;
+    if (ep_buf && ep_bytes >= trap_ep_bytes(S)) {   // the caller's buffer (pm_local_search_ep/_sigma_async)
+      if (ep_ready) {
+        ldp = trap_ep_ld(S);                         // built with E (pm_error_matrix_sigma)
+      } else {
+        const pm_status_t se = trap_build_ep_into(E, ldE, S, st, ep_buf, &ldp);
+        if (se != PM_OK) return se;
+      }
       Ep_use = ep_buf;
     } else {
       int32_t* Ep = nullptr;

@@ -839,6 +839,12 @@ pm_status_t trap_build_ep_into(const int32_t* E, int64_t ldE, int32_t S, cudaStr
   return PM_OK;
 }
 
+bool trap_ep_wanted(int32_t S) {
+  const int32_t ep_mode = knob("trap_ep", 1);
+  if (ep_mode == 0 || S < 2) return false;
+  return ep_mode == 2 || trap_ep_bytes(S) <= device_total_mem() / 8;
+}
+
 pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t** Ep,
                           int64_t* ldp) {
   *Ep = nullptr;

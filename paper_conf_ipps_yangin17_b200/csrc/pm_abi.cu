@@ -213,6 +213,39 @@ pm_status_t pm_error_matrix_tiles(const uint8_t* d_input_tiles, const uint8_t* d
   return PM_OK;
 }
 
+// Steps 1-2 for rows [row_begin, row_end), and (Ep != NULL) TRAP's
+// sigma-permuted copy of those rows in the same pass (arguments validated by
+// the callers).
+static pm_status_t error_matrix_impl(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M,
+                                     int32_t C, int32_t row_begin, int32_t row_end, int32_t* d_E, int64_t ld_E,
+                                     cudaStream_t st, int32_t* Ep) {
+  const int32_t g = N / M;
+  const int32_t S = g * g;
+  const int64_t ldp = Ep ? trap_ep_ld(S) : 0;
+  const int32_t nrows = row_end - row_begin;
+  // split-K plans accumulate E with atomics: the copy is permuted afterwards
+  const bool split = Ep && sad_split_plan(nrows, S, M * M * C);
+  int32_t* Ep_k = split ? nullptr : Ep;
+  // Step 1 fused into the E loader where the two pack launches would cost more
+  // than the loader's per-stage address arithmetic (measured: fused ~8 % slower
+  // per pair at S >= 16384, pack overhead dominant at S <= 4096).
+  if (S <= 4096 && sad_image_ok(d_input, d_target, N, M, C)) {
+    PM_CUDA_TRY(launch_sad_image(d_input, d_target, N, M, C, row_begin, row_end, d_E, ld_E, st, Ep_k, ldp));
+  } else {
+    const int64_t ldt = pm_tile_stride(M, C);
+    DevBuf buf;
+    buf.st = st;
+    PM_CUDA_TRY(pm::scratch_alloc(&buf.p, (size_t)ldt * ((size_t)nrows + S), st));
+    uint8_t* tI = reinterpret_cast<uint8_t*>(buf.p);
+    uint8_t* tT = tI + (size_t)ldt * nrows;
+    PM_CUDA_TRY(launch_pack(d_input, N, M, C, tI, ldt, row_begin, row_end, st));
+    PM_CUDA_TRY(launch_pack(d_target, N, M, C, tT, ldt, 0, S, st));
+    PM_CUDA_TRY(launch_sad(tI, tT, ldt, nrows, S, M * M * C, d_E, ld_E, st, Ep_k, ldp, row_begin));
+  }
+  if (split) PM_CUDA_TRY(launch_permute_cols(d_E, ld_E, Ep + (int64_t)row_begin * ldp, ldp, nrows, S - 1, 48, st));
+  return PM_OK;
+}
+
 pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M, int32_t C,
                             int32_t row_begin, int32_t row_end, int32_t* d_E, int64_t ld_E,
                             pm_stream_t stream) {
@@ -222,25 +255,19 @@ pm_status_t pm_error_matrix(const uint8_t* d_input, const uint8_t* d_target, int
   if (row_begin < 0 || row_end > S || row_begin > row_end || ld_E < S) return PM_ERR_INVALID;
   if (row_begin == row_end) return PM_OK;   // empty shard: nothing to do, pointers unused
   if (!d_input || !d_target || !d_E) return PM_ERR_INVALID;
-  cudaStream_t st = (cudaStream_t)stream;
-  // Step 1 fused into the E loader where the two pack launches would cost more
-  // than the loader's per-stage address arithmetic (measured: fused ~8 % slower
-  // per pair at S >= 16384, pack overhead dominant at S <= 4096).
-  if (S <= 4096 && sad_image_ok(d_input, d_target, N, M, C)) {
-    PM_CUDA_TRY(launch_sad_image(d_input, d_target, N, M, C, row_begin, row_end, d_E, ld_E, st));
-    return PM_OK;
-  }
-  const int64_t ldt = pm_tile_stride(M, C);
-  const int32_t nrows = row_end - row_begin;
-  DevBuf buf;
-  buf.st = st;
-  PM_CUDA_TRY(pm::scratch_alloc(&buf.p, (size_t)ldt * ((size_t)nrows + S), st));
-  uint8_t* tI = reinterpret_cast<uint8_t*>(buf.p);
-  uint8_t* tT = tI + (size_t)ldt * nrows;
-  PM_CUDA_TRY(launch_pack(d_input, N, M, C, tI, ldt, row_begin, row_end, st));
-  PM_CUDA_TRY(launch_pack(d_target, N, M, C, tT, ldt, 0, S, st));
-  PM_CUDA_TRY(launch_sad(tI, tT, ldt, nrows, S, M * M * C, d_E, ld_E, st));
-  return PM_OK;
+  return error_matrix_impl(d_input, d_target, N, M, C, row_begin, row_end, d_E, ld_E, (cudaStream_t)stream,
+                           nullptr);
+}
+
+pm_status_t pm_error_matrix_sigma(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M,
+                                  int32_t C, int32_t* d_E, int64_t ld_E, int32_t* d_Ep, size_t ep_bytes,
+                                  pm_stream_t stream) {
+  if (!valid_image_args(N, M, C)) return PM_ERR_INVALID;
+  const int32_t g = N / M;
+  const int32_t S = g * g;
+  if (!d_input || !d_target || !d_E || !d_Ep || ld_E < S || ep_bytes < trap_ep_bytes(S)) return PM_ERR_INVALID;
+  if (S < 2 || (S & 1)) return PM_ERR_UNSUPPORTED;   // the copy is defined for m = S-1 odd
+  return error_matrix_impl(d_input, d_target, N, M, C, 0, S, d_E, ld_E, (cudaStream_t)stream, d_Ep);
 }
 
 int32_t pm_num_colors(int32_t S) { return Classes(S).ncls; }
@@ -310,6 +337,23 @@ pm_status_t pm_local_search_ep_async(const int32_t* d_E, int64_t ld_E, int32_t S
   int32_t used = method;
   return run_local_search(d_E, ld_E, S, d_perm, max_rounds, method, reinterpret_cast<LsResult*>(d_result),
                           nullptr, 0, st, &used, d_Ep, ep_bytes);
+}
+
+pm_status_t pm_local_search_sigma_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
+                                        int32_t max_rounds, int32_t method, const int32_t* d_Ep, size_t ep_bytes,
+                                        int64_t* d_result, pm_stream_t stream) {
+  if (!d_result || !d_Ep || ep_bytes < trap_ep_bytes(S) || !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method))
+    return PM_ERR_INVALID;
+  {
+    const pm_status_t v = ls_method_supported(S, method);
+    if (v != PM_OK) return v;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  PM_CUDA_TRY(cudaMemsetAsync(d_result, 0, sizeof(LsResult), st));
+  int32_t used = method;
+  // (the copy is only read: ep_ready)
+  return run_local_search(d_E, ld_E, S, d_perm, max_rounds, method, reinterpret_cast<LsResult*>(d_result),
+                          nullptr, 0, st, &used, const_cast<int32_t*>(d_Ep), ep_bytes, true);
 }
 
 size_t pm_trap_workspace_bytes(int32_t S) { return (S < 2) ? 0 : trap_ws_bytes(S); }
@@ -478,11 +522,26 @@ pm_status_t pm_photomosaic_async(const uint8_t* d_input, const uint8_t* d_target
     if (v != PM_OK) return v;
   }
   cudaStream_t st = (cudaStream_t)stream;
-  pm_status_t s = pm_error_matrix(d_input, d_target, N, M, C, 0, S, d_E, ld_E, stream);   // Steps 1-2
-  if (s != PM_OK) return s;
-  PM_CUDA_TRY(launch_iota(d_perm, S, st));                                                // r = identity
-  s = pm_local_search_async(d_E, ld_E, S, d_perm, 0, method, d_result, stream);           // Alg. 2
-  if (s != PM_OK) return s;
+  // TRAP stages from the sigma-permuted copy of E: write it in the E pass
+  // (pm_error_matrix_sigma) when the search would build it anyway
+  const int32_t used = method == PM_LS_AUTO ? pm_ls_auto_method(S) : method;
+  ScopedScratch ep(st);
+  if (used == PM_LS_TRAP && trap_ep_wanted(S)) {
+    PM_CUDA_TRY(pm::scratch_alloc(&ep.p, trap_ep_bytes(S), st));
+    pm_status_t s = pm_error_matrix_sigma(d_input, d_target, N, M, C, d_E, ld_E, ep.as<int32_t>(),
+                                          trap_ep_bytes(S), stream);                        // Steps 1-2 (+ copy)
+    if (s != PM_OK) return s;
+    PM_CUDA_TRY(launch_iota(d_perm, S, st));                                                // r = identity
+    s = pm_local_search_sigma_async(d_E, ld_E, S, d_perm, 0, method, ep.as<int32_t>(), trap_ep_bytes(S),
+                                    d_result, stream);                                      // Alg. 2
+    if (s != PM_OK) return s;
+  } else {
+    pm_status_t s = pm_error_matrix(d_input, d_target, N, M, C, 0, S, d_E, ld_E, stream);   // Steps 1-2
+    if (s != PM_OK) return s;
+    PM_CUDA_TRY(launch_iota(d_perm, S, st));                                                // r = identity
+    s = pm_local_search_async(d_E, ld_E, S, d_perm, 0, method, d_result, stream);           // Alg. 2
+    if (s != PM_OK) return s;
+  }
   PM_CUDA_TRY(launch_cost(d_E, ld_E, S, d_perm, d_result + 3, st));                       // Eq. (2)
   return PM_OK;
 }

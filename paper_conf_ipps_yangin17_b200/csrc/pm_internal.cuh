@@ -101,15 +101,21 @@ struct Classes {
 // Internal launchers (defined in k_sad.cu / k_search.cu).
 cudaError_t launch_pack(const uint8_t* img, int32_t N, int32_t M, int32_t C, uint8_t* tiles,
                         int64_t ld_tiles, int32_t tile_begin, int32_t tile_end, cudaStream_t st);
+// Ep (optional): also write TRAP's sigma-permuted copy Ep[row0 + r][sigma(v)]
+// (+ its cyclic extension) in the epilogue -- only when the plan has no
+// split-K (sad_split_plan false); the caller permutes E afterwards otherwise.
 cudaError_t launch_sad(const uint8_t* A, const uint8_t* B, int64_t ldt, int32_t nrows, int32_t S,
-                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st);
+                       int32_t P, int32_t* E, int64_t ldE, cudaStream_t st, int32_t* Ep = nullptr,
+                       int64_t ldp = 0, int32_t row0 = 0);
+bool sad_split_plan(int32_t nrows, int32_t S, int32_t P);
 cudaError_t launch_render(const uint8_t* img, int32_t N, int32_t M, int32_t C, const int32_t* perm,
                           uint8_t* out, cudaStream_t st);
 // Step 1 fused into the E kernel's loader (no packed tiles): requires
 // sad_image_ok (a tile row is a whole number of 16-byte pieces, P % 64 == 0).
 bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C);
 cudaError_t launch_sad_image(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C,
-                             int32_t row_begin, int32_t row_end, int32_t* E, int64_t ldE, cudaStream_t st);
+                             int32_t row_begin, int32_t row_end, int32_t* E, int64_t ldE, cudaStream_t st,
+                             int32_t* Ep = nullptr, int64_t ldp = 0);
 
 // Device-side result of one search; layout = the int64 [3] of
 // pm_local_search_async's d_result: {status, rounds, swaps}.
@@ -124,7 +130,8 @@ cudaError_t launch_iota(int32_t* perm, int32_t S, cudaStream_t st);
 pm_status_t run_local_search(const int32_t* E, int64_t ldE, int32_t S, int32_t* perm,
                              int32_t max_rounds, int32_t method, LsResult* dev_out,
                              int64_t* dev_per_round, int32_t max_log, cudaStream_t st,
-                             int32_t* used_method, int32_t* ep_buf = nullptr, size_t ep_bytes = 0);
+                             int32_t* used_method, int32_t* ep_buf = nullptr, size_t ep_bytes = 0,
+                             bool ep_ready = false);
 int32_t ls_class_launches_per_round(int32_t S);
 int32_t ls_window_max_S();
 // Ep[t][pos] = E[t][2 pos mod m], pos in [0, m + ext) (sigma-permuted rows, k_window.cu)
@@ -222,6 +229,7 @@ pm_status_t trap_build_ep(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t
 // trap_build_ep_into (pm_local_search_ep_async).
 int64_t trap_ep_ld(int32_t S);
 size_t trap_ep_bytes(int32_t S);
+bool trap_ep_wanted(int32_t S);   // would trap_build_ep build the copy for S (trap_ep rule)?
 pm_status_t trap_build_ep_into(const int32_t* E, int64_t ldE, int32_t S, cudaStream_t st, int32_t* Ep, int64_t* ldp);
 
 // Multi-rank TRAP (k_trap.cu).

@@ -41,6 +41,8 @@ _SIGS = [
     ("pm_local_search_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, _P]),
     ("pm_sigma_copy_bytes", ctypes.c_size_t, [_I32]),
     ("pm_local_search_ep_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, ctypes.c_size_t, _P, _P]),
+    ("pm_error_matrix_sigma", ctypes.c_int, [_P, _P, _I32, _I32, _I32, _P, _I64, _P, ctypes.c_size_t, _P]),
+    ("pm_local_search_sigma_async", ctypes.c_int, [_P, _I64, _I32, _P, _I32, _I32, _P, ctypes.c_size_t, _P, _P]),
     ("pm_ls_auto_method", _I32, [_I32]),
     ("pm_init_identity", ctypes.c_int, [_P, _I32, _P]),
     ("pm_cost", ctypes.c_int, [_P, _I64, _I32, _P, _P, _P]),
@@ -235,6 +237,26 @@ def local_search_ep_async(E, perm, result, Ep, max_rounds: int = 0, method: str 
                                           METHODS[method], Ep.data_ptr(), Ep.numel() * Ep.element_size(),
                                           result.data_ptr(), _stream(stream)),
            "pm_local_search_ep_async")
+
+
+def error_matrix_sigma(I, T, M: int, E, Ep, stream=None):
+    """pm_error_matrix_sigma: E (all rows) and its sigma-permuted copy Ep in one pass."""
+    torch = _torch()
+    I = _dev_u8_image(I)
+    T = _dev_u8_image(T)
+    _dev(E, torch.int32)
+    _check(lib().pm_error_matrix_sigma(I.data_ptr(), T.data_ptr(), I.shape[0], M, I.shape[2], E.data_ptr(),
+                                       E.stride(0), Ep.data_ptr(), Ep.numel() * Ep.element_size(), _stream(stream)),
+           "pm_error_matrix_sigma")
+    return E
+
+
+def local_search_sigma_async(E, perm, result, Ep, max_rounds: int = 0, method: str = "auto", stream=None):
+    """pm_local_search_sigma_async: as local_search_async on a prebuilt sigma-permuted copy Ep."""
+    _check(lib().pm_local_search_sigma_async(E.data_ptr(), E.stride(0), E.shape[0], perm.data_ptr(), max_rounds,
+                                             METHODS[method], Ep.data_ptr(), Ep.numel() * Ep.element_size(),
+                                             result.data_ptr(), _stream(stream)),
+           "pm_local_search_sigma_async")
 
 
 def local_search_multi_emulated(E, world: int, perm=None, max_rounds: int = 0, stream=None):

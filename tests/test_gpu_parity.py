@@ -884,3 +884,51 @@ def test_local_search_caller_owned_sigma_copy_too_small_rejected():
     with pytest.raises(pm.PMError) as e:
         pm.local_search_ep_async(E, perm, res, Ep, method="trap")
     assert e.value.status == pm.PM_ERR_INVALID
+
+
+# ---- pm_error_matrix_sigma: E and its sigma-permuted copy in one pass (the
+# E kernel's epilogue writes both), and pm_local_search_sigma_async on it
+def _sigma_ref(E_np):
+    S = E_np.shape[0]
+    m = S - 1
+    q = np.arange(m + 48)
+    return E_np[:, (2 * q) % m]
+
+
+@pytest.mark.parametrize("N,M,C,fam,plan", [(128, 8, 3, "smooth", 0), (512, 16, 3, "noise", 0), (1024, 16, 3, "smooth", 0),
+                                            (512, 16, 3, "smooth", 128002), (512, 16, 3, "ties", 64003),
+                                            (256, 16, 1, "smooth", 0), (160, 10, 3, "noise", 0)])
+def test_error_matrix_sigma_parity(N, M, C, fam, plan):
+    # plan: sad_plan override (split-K plans accumulate E atomically, so the
+    # copy is permuted from E afterwards instead of in the epilogue)
+    if plan:
+        pm.tuning_set("sad_plan", plan)
+    I, T = pair(fam, N, M, C)
+    E_np = oracle_E(fam, N, M, C)
+    S = E_np.shape[0]
+    nbytes = pm.sigma_copy_bytes(S)
+    E = torch.full((S, S), -1, dtype=torch.int32, device=DEV)
+    Ep = torch.full((nbytes // 4,), -7, dtype=torch.int32, device=DEV)
+    pm.error_matrix_sigma(dev(I), dev(T), M, E, Ep)
+    torch.cuda.synchronize()
+    assert (E.cpu().numpy() == E_np).all()
+    ld = nbytes // 4 // S
+    assert (Ep.view(S, ld)[:, : S - 1 + 48].cpu().numpy() == _sigma_ref(E_np)).all()
+    # the search on the prebuilt copy gives the oracle's replay
+    ref = oracle.local_search(E_np)
+    perm = torch.arange(S, dtype=torch.int32, device=DEV)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    pm.local_search_sigma_async(E, perm, res, Ep)
+    torch.cuda.synchronize()
+    assert res.cpu().tolist() == [ref[4], ref[1], ref[2]]
+    assert (perm.cpu().numpy() == ref[0]).all()
+
+
+def test_error_matrix_sigma_odd_S_unsupported():
+    I, T = pair("smooth", 90, 10, 3)   # S = 81
+    S = 81
+    E = torch.empty((S, S), dtype=torch.int32, device=DEV)
+    Ep = torch.empty(max(pm.sigma_copy_bytes(S) // 4, 1), dtype=torch.int32, device=DEV)
+    with pytest.raises(pm.PMError) as e:
+        pm.error_matrix_sigma(dev(I), dev(T), 10, E, Ep)
+    assert e.value.status == pm.PM_ERR_UNSUPPORTED

@@ -109,6 +109,32 @@ def test_cfg4_caller_owned_sigma_copy(cfg4):
     _assert_search((perm, rounds, swaps, None, st), ref, E_or, "config 4 auto, caller-owned sigma copy")
 
 
+def test_cfg4_error_matrix_sigma(cfg4):
+    # E and its sigma-permuted copy in one pass (the bench's Step 2), then the
+    # search on that copy: E equal to the oracle's, the copy equal to its
+    # permutation, the search equal to the oracle's replay
+    I, T, E_or, E_gpu, ref = cfg4
+    S = E_or.shape[0]
+    nbytes = pm.sigma_copy_bytes(S)
+    E = torch.empty((S, S), dtype=torch.int32, device=DEV)
+    Ep = torch.empty(nbytes // 4, dtype=torch.int32, device=DEV)
+    pm.error_matrix_sigma(dev(I), dev(T), 16, E, Ep)
+    _assert_E_equal(E, E_or)
+    ld = nbytes // 4 // S
+    q = np.arange(S - 1 + 48)
+    cols = (2 * q) % (S - 1)
+    Epv = Ep.view(S, ld)
+    for r0 in range(0, S, 4096):
+        assert (Epv[r0:r0 + 4096, : S - 1 + 48].cpu().numpy() == E_or[r0:r0 + 4096][:, cols]).all()
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    perm = torch.arange(S, dtype=torch.int32, device=DEV)
+    pm.local_search_sigma_async(E, perm, res, Ep)
+    st, rounds, swaps = res.cpu().tolist()
+    _assert_search((perm, rounds, swaps, None, st), ref, E_or, "config 4 auto on the fused sigma copy")
+    del E, Ep
+    torch.cuda.empty_cache()
+
+
 def test_cfg4_trap_every_round(cfg4):
     # the sparse hand-over off: every round (incl. the quiet ones) on TRAP
     I, T, E_or, E_gpu, ref = cfg4
