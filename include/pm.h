@@ -179,22 +179,25 @@ pm_status_t pm_local_search_async(const int32_t* d_E, int64_t ld_E, int32_t S, i
  *               16-byte aligned, owned by the caller; overwritten (any other
  *               method leaves it untouched).
  * Results are identical to pm_local_search_async (Alg. 2).
- * PM_ERR_INVALID for a NULL or too small d_Ep, else as pm_local_search_async. */
+ * PM_ERR_INVALID for a NULL, misaligned or too small d_Ep, else as
+ * pm_local_search_async. */
 size_t pm_sigma_copy_bytes(int32_t S);
 /* Steps 1-2 (Eq. 1; all S rows) AND the sigma-permuted copy in one
  * pass: the E kernel writes each entry E[u][v] also to d_Ep[u][sigma(v)]
  * (and to d_Ep[u][sigma(v) + m] when sigma(v) < 48), saving the separate
  * read + write of E that pm_local_search_ep_async / pm_local_search_async
  * spend on it.  d_E, ld_E as pm_error_matrix (row_begin = 0, row_end = S);
- * d_Ep as pm_local_search_ep_async.  S must be even (m = S-1 odd), else
- * PM_ERR_UNSUPPORTED.  Asynchronous on `stream`. */
+ * d_Ep as pm_local_search_ep_async (16-byte aligned, PM_ERR_INVALID
+ * otherwise).  S must be even (m = S-1 odd), else PM_ERR_UNSUPPORTED.
+ * Asynchronous on `stream`. */
 pm_status_t pm_error_matrix_sigma(const uint8_t* d_input, const uint8_t* d_target, int32_t N, int32_t M,
                                   int32_t C, int32_t* d_E, int64_t ld_E, int32_t* d_Ep, size_t ep_bytes,
                                   pm_stream_t stream);
 /* pm_local_search_async on a copy d_Ep that already holds E's
  * sigma-permuted rows (from pm_error_matrix_sigma or pm_local_search_ep_async
- * on this E; read only).  A stale copy gives wrong results: the caller keeps
- * it in step with E. */
+ * on this E; read only; 16-byte aligned).  A stale copy gives wrong results:
+ * the caller keeps it in step with E.  PM_ERR_INVALID for a NULL, misaligned
+ * or too small d_Ep. */
 pm_status_t pm_local_search_sigma_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
                                         int32_t max_rounds, int32_t method, const int32_t* d_Ep, size_t ep_bytes,
                                         int64_t* d_result, pm_stream_t stream);

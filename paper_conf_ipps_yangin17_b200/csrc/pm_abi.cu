@@ -265,7 +265,9 @@ pm_status_t pm_error_matrix_sigma(const uint8_t* d_input, const uint8_t* d_targe
   if (!valid_image_args(N, M, C)) return PM_ERR_INVALID;
   const int32_t g = N / M;
   const int32_t S = g * g;
-  if (!d_input || !d_target || !d_E || !d_Ep || ld_E < S || ep_bytes < trap_ep_bytes(S)) return PM_ERR_INVALID;
+  if (!d_input || !d_target || !d_E || !d_Ep || ld_E < S || ep_bytes < trap_ep_bytes(S) ||
+      (reinterpret_cast<uintptr_t>(d_Ep) & 15))
+    return PM_ERR_INVALID;
   if (S < 2 || (S & 1)) return PM_ERR_UNSUPPORTED;   // the copy is defined for m = S-1 odd
   return error_matrix_impl(d_input, d_target, N, M, C, 0, S, d_E, ld_E, (cudaStream_t)stream, d_Ep);
 }
@@ -326,7 +328,8 @@ size_t pm_sigma_copy_bytes(int32_t S) { return trap_ep_bytes(S); }
 pm_status_t pm_local_search_ep_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
                                      int32_t max_rounds, int32_t method, int32_t* d_Ep, size_t ep_bytes,
                                      int64_t* d_result, pm_stream_t stream) {
-  if (!d_result || !d_Ep || ep_bytes < trap_ep_bytes(S) || !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method))
+  if (!d_result || !d_Ep || ep_bytes < trap_ep_bytes(S) || (reinterpret_cast<uintptr_t>(d_Ep) & 15) ||
+      !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method))
     return PM_ERR_INVALID;
   {
     const pm_status_t v = ls_method_supported(S, method);
@@ -342,7 +345,8 @@ pm_status_t pm_local_search_ep_async(const int32_t* d_E, int64_t ld_E, int32_t S
 pm_status_t pm_local_search_sigma_async(const int32_t* d_E, int64_t ld_E, int32_t S, int32_t* d_perm,
                                         int32_t max_rounds, int32_t method, const int32_t* d_Ep, size_t ep_bytes,
                                         int64_t* d_result, pm_stream_t stream) {
-  if (!d_result || !d_Ep || ep_bytes < trap_ep_bytes(S) || !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method))
+  if (!d_result || !d_Ep || ep_bytes < trap_ep_bytes(S) || (reinterpret_cast<uintptr_t>(d_Ep) & 15) ||
+      !valid_ls_args(d_E, ld_E, S, d_perm, max_rounds, method))
     return PM_ERR_INVALID;
   {
     const pm_status_t v = ls_method_supported(S, method);

@@ -932,3 +932,17 @@ def test_error_matrix_sigma_odd_S_unsupported():
     with pytest.raises(pm.PMError) as e:
         pm.error_matrix_sigma(dev(I), dev(T), 10, E, Ep)
     assert e.value.status == pm.PM_ERR_UNSUPPORTED
+
+
+def test_sigma_copy_misaligned_rejected():
+    E_np = oracle_E("smooth", 128, 8)
+    S = E_np.shape[0]
+    E = dev(E_np)
+    buf = torch.empty(pm.sigma_copy_bytes(S) // 4 + 4, dtype=torch.int32, device=DEV)
+    Ep = buf[1:1 + pm.sigma_copy_bytes(S) // 4]   # 4-byte offset: not 16-byte aligned
+    perm = torch.arange(S, dtype=torch.int32, device=DEV)
+    res = torch.zeros(3, dtype=torch.int64, device=DEV)
+    for call in (lambda: pm.local_search_ep_async(E, perm, res, Ep), lambda: pm.local_search_sigma_async(E, perm, res, Ep)):
+        with pytest.raises(pm.PMError) as e:
+            call()
+        assert e.value.status == pm.PM_ERR_INVALID
