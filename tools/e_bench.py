@@ -19,7 +19,10 @@ for cfg in cfgs:
     dI, dT = torch.from_numpy(I).cuda(), torch.from_numpy(T).cuda()
     E = torch.empty((S, S), dtype=torch.int32, device="cuda")
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
-    for variant in ("fused", "packed"):
+    Ep = torch.empty(pm.sigma_copy_bytes(S) // 4, dtype=torch.int32, device="cuda") if S % 2 == 0 else None
+    for variant in ("fused", "packed", "sigma"):
+        if variant == "sigma" and Ep is None:
+            continue
         ts = []
         It = Tt = None
         if variant == "packed":
@@ -30,6 +33,8 @@ for cfg in cfgs:
             a.record()
             if variant == "fused":
                 pm.error_matrix(dI, dT, M, out=E)
+            elif variant == "sigma":   # E + the sigma-permuted copy in one pass
+                pm.error_matrix_sigma(dI, dT, M, E, Ep)
             else:
                 pm.error_matrix_tiles(It, Tt, P, out=E)
             b.record()
@@ -40,5 +45,5 @@ for cfg in cfgs:
         ops = S * S * P / (ms * 1e-3)
         print(f"cfg{cfg} S={S:6d} P={P} {variant:6s} {ms:9.3f} ms  {S*S/(ms*1e-3)/1e9:8.2f} Gpairs/s  "
               f"{ops/1e12:6.2f} T absdiff/s = {100*ops/PEAK:5.1f}% of ALU peak @1965MHz", flush=True)
-    del E
+    del E, Ep
     torch.cuda.empty_cache()
