@@ -6,17 +6,22 @@
 // threshold-decomposition form would need 255x the MACs; DESIGN.md "E
 // kernel").  It runs on the integer ALU pipe instead: one
 // `vabsdiff4.u32.u32.u32.add` (SASS VABSDIFF4.U8.ACC) consumes 4 byte pairs
-// and accumulates into an int32, and issues at the IADD3 rate (64/clk/SM,
-// tools/ubench_alu.cu).  The kernel is a register-blocked "SAD-GEMM":
-//   * CTA tile 128 (input tiles u) x 128 (target tiles v), 256 threads, each
-//     thread 8 x 8 outputs (128 x 64 and 8 x 4, two CTAs per SM, for small S) (rows ty + 16 i, cols tx + 16 j -> conflict-free
-//     LDS.128 on a 80-byte padded smem row stride);
+// and accumulates into an int32; it issues at 64 /clk/SM, half the IADD3
+// rate (~124 /clk/SM in the same microbenchmark, tools/ubench_alu.cu,
+// profiles/r01_ubench_alu.txt).  The kernel is a register-blocked "SAD-GEMM":
+//   * CTA tile 128 (input tiles u) x 64 (target tiles v), 256 threads, each
+//     thread 8 x 4 outputs, two CTAs per SM (the 128 x 128 / 8 x 8 variant
+//     measured ~3 % slower at every size); rows ty + 16 i, cols tx + 16 j ->
+//     conflict-free LDS.128 on a 80-byte padded smem row stride;
 //   * K (the P bytes of a tile) streamed in 64-byte chunks through a 4-stage
 //     cp.async.cg ring (16-byte copies, L2-only), so smem holds 16 words per
 //     row per stage;
-//   * per 4 K-words a thread issues 16 LDS.128 and 256 VABSDIFF4 (16:1);
-//   * split-K over gridDim.z for small S (integer red.add is exact and
-//     order-independent), chosen on the host to fill all 148 SMs.
+//   * per 4 K-words a thread issues 12 LDS.128 and 128 VABSDIFF4 (8 x 8 tile: 16 and 256);
+//   * split-K over gridDim.z available (integer red.add is exact and
+//     order-independent), chosen on the host only when it pays (measured:
+//     never at configs 1-5);
+//   * optionally the epilogue also writes TRAP's sigma-permuted copy of E
+//     (pm_error_matrix_sigma).
 #include "pm_internal.cuh"
 
 namespace pm {
