@@ -139,6 +139,7 @@ struct SadGeom {
   int32_t a_tile0;         // image: tile index of local row 0 (row_begin)
   int32_t g, M, R, MC;     // image: tiles per grid row, tile side, pieces per tile row, M*C
   int32_t e_row0;          // row of Ep that local row 0 goes to (the sigma copy, when written)
+  int32_t vec_out;         // 0: scalar epilogue; >= 1: E rows 16-byte aligned (staged epilogue); 2: also S/2 % 4 == 0
 };
 
 template <bool kImage>
@@ -246,6 +247,57 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
   }
   cp_async_wait<0>();
 
+  // Full tiles with 16-byte-aligned rows (geo.vec_out): the outputs go
+  // through shared memory and leave as coalesced 16-byte stores -- E's rows,
+  // and the sigma copy's two contiguous runs per row (even columns -> q =
+  // col/2, odd -> (col + m)/2 = col/2 + S/2) -- instead of one 4-byte store
+  // per entry (and two per entry of the copy).
+  const int32_t mq = S - 1;
+  if (!kAtomic && geo.vec_out && row0 + BM <= nrows && col0 + BN < S) {   // (col0 + BN <= m: every column in the copy)
+    constexpr int OS = BN + 16;                         // padded row stride: conflict-free fills
+    static_assert(BM * OS * 4 <= kStages * (BM + BN) * ROWW * 4, "staged tile fits the pipeline smem");
+    __syncthreads();                                    // every warp done with the pipeline buffers
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) smem[(ty + 16 * i) * OS + tx + 16 * j] = acc[i][j];
+    __syncthreads();
+    constexpr int NV = BM * BN / 4 / kThreads;          // 16-byte pieces per thread
+#pragma unroll
+    for (int v = 0; v < NV; ++v) {
+      const int idx = tid + v * kThreads;
+      const int r = idx / (BN / 4), c4 = idx - r * (BN / 4);
+      const uint4 val = *reinterpret_cast<const uint4*>(smem + r * OS + 4 * c4);
+      *reinterpret_cast<uint4*>(E + (int64_t)(row0 + r) * ldE + col0 + 4 * c4) = val;
+    }
+    if (Ep) {
+      const bool odd_vec = geo.vec_out > 1;             // S/2 % 4 == 0: the odd run is 16-byte aligned too
+#pragma unroll
+      for (int v = 0; v < NV; ++v) {
+        const int idx = tid + v * kThreads;
+        const int r = idx / (BN / 4), w = idx - r * (BN / 4);
+        const int par = w >= BN / 8 ? 1 : 0, k4 = w - par * (BN / 8);
+        const uint32_t* srow = smem + r * OS + 8 * k4 + par;
+        const uint4 val = make_uint4(srow[0], srow[2], srow[4], srow[6]);
+        const int32_t q0 = (col0 >> 1) + (par ? (S >> 1) : 0) + 4 * k4;
+        int32_t* prow = Ep + (int64_t)(geo.e_row0 + row0 + r) * ldp;
+        if (!par || odd_vec) {
+          *reinterpret_cast<uint4*>(prow + q0) = val;
+        } else {
+          prow[q0] = (int32_t)val.x; prow[q0 + 1] = (int32_t)val.y;
+          prow[q0 + 2] = (int32_t)val.z; prow[q0 + 3] = (int32_t)val.w;
+        }
+        if (q0 < 48) {                                  // the cyclic extension, q + m for q < 48
+          const uint32_t vv[4] = {val.x, val.y, val.z, val.w};
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            if (q0 + e < 48) prow[q0 + e + mq] = (int32_t)vv[e];
+        }
+      }
+    }
+    return;
+  }
+
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
     const int32_t row = row0 + ty + 16 * i;
@@ -343,6 +395,10 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
   if (gy > 65535) return cudaErrorInvalidValue;
   const SadPlan plan = choose_plan(nrows, S, nkb, sms);
   const int split = plan.split;
+  SadGeom g2 = geo;
+  g2.vec_out = ((ldE & 3) == 0 && (reinterpret_cast<uintptr_t>(E) & 15) == 0 &&
+                (!Ep || (reinterpret_cast<uintptr_t>(Ep) & 15) == 0))
+                   ? (((S / 2) % 4 == 0) ? 2 : 1) : 0;
   if (split > 1) {
     // split-K accumulates with red.add: zero the [nrows][S] window of E first
     cudaError_t e = (ldE == S)
@@ -353,22 +409,22 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
   if (plan.bn == 64) {
     dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, (unsigned)split);
     if (split > 1) {
-      if (image) k_sad<true, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
-      else k_sad<true, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
+      if (image) k_sad<true, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
+      else k_sad<true, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
     } else {
-      if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
-      else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
+      if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
+      else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
     }
     note_launch();
     return cudaGetLastError();
   }
   dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
   if (split > 1) {   // (split-K accumulates: the sigma copy follows E, launch_sad_sigma)
-    if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
-    else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw / split, E, ldE, nullptr, 0);
+    if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
+    else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
   } else {
-    if (image) k_sad<false, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
-    else k_sad<false, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(geo, nrows, S, kw, E, ldE, Ep, ldp);
+    if (image) k_sad<false, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
+    else k_sad<false, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
   }
   note_launch();
   return cudaGetLastError();
