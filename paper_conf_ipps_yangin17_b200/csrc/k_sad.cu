@@ -291,7 +291,7 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
           const uint32_t vv[4] = {val.x, val.y, val.z, val.w};
 #pragma unroll
           for (int e = 0; e < 4; ++e)
-            if (q0 + e < 48) prow[q0 + e + mq] = (int32_t)vv[e];
+            for (int32_t qq = q0 + e + mq; qq < mq + 48; qq += mq) prow[qq] = (int32_t)vv[e];
         }
       }
     }
@@ -312,15 +312,15 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
       // the sigma-permuted copy TRAP stages from (k_trap.cu), written in the
       // same pass (no separate read + write of E): Ep[row][q] = E[row][2q mod m]
       // for q < m + 48 cyclic, m = S - 1 odd -> column col lands at
-      // q = sigma(col) = col/2 (even) or (col+m)/2 (odd), and again at q + m
-      // when q < 48
+      // q = sigma(col) = col/2 (even) or (col+m)/2 (odd), and again at q + m,
+      // q + 2m, ... below m + 48
       if (!kAtomic && Ep) {
         const int32_t m = S - 1;
         if (col < m) {
           const int32_t q = (col & 1) ? (col + m) >> 1 : col >> 1;
           int32_t* prow = Ep + (int64_t)(geo.e_row0 + row) * ldp;
           prow[q] = (int32_t)acc[i][j];
-          if (q < 48) prow[q + m] = (int32_t)acc[i][j];
+          for (int32_t qq = q + m; qq < m + 48; qq += m) prow[qq] = (int32_t)acc[i][j];   // (m < 48: wraps again)
         }
       }
     }

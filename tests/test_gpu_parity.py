@@ -897,7 +897,8 @@ def _sigma_ref(E_np):
 
 @pytest.mark.parametrize("N,M,C,fam,plan", [(128, 8, 3, "smooth", 0), (512, 16, 3, "noise", 0), (1024, 16, 3, "smooth", 0),
                                             (512, 16, 3, "smooth", 128002), (512, 16, 3, "ties", 64003),
-                                            (256, 16, 1, "smooth", 0), (160, 10, 3, "noise", 0)])
+                                            (256, 16, 1, "smooth", 0), (160, 10, 3, "noise", 0),
+                                            (48, 8, 3, "noise", 0), (32, 8, 1, "smooth", 0)])   # m < 48: the extension wraps twice
 def test_error_matrix_sigma_parity(N, M, C, fam, plan):
     # plan: sad_plan override (split-K plans accumulate E atomically, so the
     # copy is permuted from E afterwards instead of in the epilogue)
