@@ -7,6 +7,8 @@ import torch
 from paper_conf_ipps_yangin17_b200 import pm, synth
 sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 import _devknobs  # noqa: E402
+if os.environ.get("PM_LIB"):   # a development build of the library
+    pm.LIB_PATH = os.environ["PM_LIB"]
 _devknobs.apply(pm)
 
 PEAK = 148 * 64 * 4 * 1.965e9          # VABSDIFF4.U8.ACC: 64 /clk/SM, 4 byte-absdiffs each
