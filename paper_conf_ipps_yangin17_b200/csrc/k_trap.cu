@@ -630,7 +630,8 @@ k_ls_trap(const TrapParams p) {
         if (prof) { const unsigned long long t = gtimer(); t_pub += t - tq; }
         group_sync(1 + grp, GT);
         if (!CLU && p.nbsync && have && gt == 0) {   // this chunk's slots of phase qph are out
-          __threadfence();
+          // (the release is cumulative: the group's publish stores happen
+          // before it through the barrier above)
           asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p.flags + ch), "r"(qph + 1u) : "memory");
         }
       }
