@@ -13,9 +13,9 @@
 //     thread 8 x 4 outputs, two CTAs per SM (the 128 x 128 / 8 x 8 variant
 //     measured ~3 % slower at every size); rows ty + 16 i, cols tx + 16 j ->
 //     conflict-free LDS.128 on a 80-byte padded smem row stride;
-//   * K (the P bytes of a tile) streamed in 64-byte chunks through a 4-stage
-//     cp.async.cg ring (16-byte copies, L2-only), so smem holds 16 words per
-//     row per stage;
+//   * K (the P bytes of a tile) streamed in 128-byte chunks (64 when K is not
+//     a multiple of 32 words) through a 4-stage cp.async.cg ring (16-byte
+//     copies, L2-only): 6 main-loop iterations per tile at P = 768;
 //   * per 4 K-words a thread issues 12 LDS.128 and 128 VABSDIFF4 (8 x 8 tile: 16 and 256);
 //   * split-K over gridDim.z available (integer red.add is exact and
 //     order-independent), chosen on the host only when it pays (measured:
@@ -104,11 +104,15 @@ cudaError_t launch_render(const uint8_t* img, int32_t N, int32_t M, int32_t C, c
 namespace sad {
 constexpr int kThreads = 256;
 constexpr int BM = 128;          // tile rows (input tiles u); BN (target tiles v) is 128 or 64
-constexpr int BKW = 16;          // K words (4 bytes each) per pipeline stage
 constexpr int kStages = 4;
-constexpr int ROWW = BKW + 4;    // padded smem row stride in words (80 B)
-template <int BN>
-constexpr int smem_bytes() { return kStages * (BM + BN) * ROWW * 4; }   // 80 / 60 KiB
+// K words (4 bytes each) per pipeline stage: 32 when K is a multiple of 32
+// words (P = 768: 6 instead of 12 main-loop iterations per tile, each with
+// its barrier and copy issue -- config 4 E 3.47 -> 3.26 ms, 80 -> 85 % of the
+// ALU peak), else 16.  Padded smem row stride KW + 4 words (conflict-free
+// LDS.128 for both).
+template <int BN, int KW>
+constexpr int smem_bytes() { return kStages * (BM + BN) * (KW + 4) * 4; }   // 60 / 110 KiB at BN = 64
+inline int stage_words(int64_t kw) { return (kw % 32 == 0) ? 32 : 16; }
 }  // namespace sad
 
 __device__ __forceinline__ uint32_t sad4(uint32_t a, uint32_t b, uint32_t c) {
@@ -155,11 +159,13 @@ __device__ __forceinline__ const uint8_t* sad_tile_base(const SadGeom& geo, cons
 // handled by one blockIdx.z slice.  BN = 128: 8 x 8 outputs per thread, one
 // CTA per SM; BN = 64: 8 x 4, two CTAs per SM (for grids too small to fill
 // 148 SMs with 128 x 128 tiles without split-K).
-template <bool kAtomic, bool kImage, int BN>
+template <bool kAtomic, bool kImage, int BN, int KW>
 __global__ void __launch_bounds__(sad::kThreads, BN == 128 ? 1 : 2)
 k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restrict__ E, int64_t ldE,
       int32_t* __restrict__ Ep, int64_t ldp) {
   using namespace sad;
+  constexpr int BKW = KW;                              // K words per pipeline stage
+  constexpr int ROWW = KW + 4;                         // padded smem row stride in words
   constexpr int NJ = BN / 16;                          // output columns per thread
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t* sA = smem;                                 // [kStages][BM][ROWW]
@@ -171,20 +177,22 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
   const int32_t piece0 = blockIdx.z * kw_split / 4;    // first 16-byte piece of this K slice
   const int nkb = kw_split / BKW;
 
-  // Loader: per stage, BM (BN) rows x 64 B = 4 BM (4 BN) 16-byte pieces per
-  // operand; thread tid copies pieces q = tid + h * 256 (row q >> 2, part q & 3).
-  constexpr int HA = BM * 4 / kThreads, HB = BN * 4 / kThreads;
+  // Loader: per stage, BM (BN) rows x 4 BKW B = PPR BM (PPR BN) 16-byte
+  // pieces per operand (PPR = BKW / 4); thread tid copies pieces
+  // q = tid + h * 256 (row q / PPR, part q % PPR).
+  constexpr int PPR = BKW / 4;
+  constexpr int HA = BM * PPR / kThreads, HB = BN * PPR / kThreads;
   const uint8_t* baseA[HA];
   const uint8_t* baseB[HB];
-  const int part = tid & 3;
+  const int part = tid % PPR;
 #pragma unroll
   for (int h = 0; h < HA; ++h) {
-    int32_t ra = row0 + ((tid + h * kThreads) >> 2); if (ra >= nrows) ra = nrows - 1;   // clamp: loaded, never stored
+    int32_t ra = row0 + (tid + h * kThreads) / PPR; if (ra >= nrows) ra = nrows - 1;   // clamp: loaded, never stored
     baseA[h] = sad_tile_base<kImage>(geo, geo.A, kImage ? geo.a_tile0 + ra : ra);
   }
 #pragma unroll
   for (int h = 0; h < HB; ++h) {
-    int32_t rb = col0 + ((tid + h * kThreads) >> 2); if (rb >= S) rb = S - 1;
+    int32_t rb = col0 + (tid + h * kThreads) / PPR; if (rb >= S) rb = S - 1;
     baseB[h] = sad_tile_base<kImage>(geo, geo.B, rb);
   }
   auto load_stage = [&](int kb, int stage) {
@@ -197,9 +205,9 @@ k_sad(SadGeom geo, int32_t nrows, int32_t S, int32_t kw_split, int32_t* __restri
       off = (int64_t)p * 16;
     }
 #pragma unroll
-    for (int h = 0; h < HA; ++h) cp_async16(sA + stage * BM * ROWW + ((tid + h * kThreads) >> 2) * ROWW + part * 4, baseA[h] + off);
+    for (int h = 0; h < HA; ++h) cp_async16(sA + stage * BM * ROWW + ((tid + h * kThreads) / PPR) * ROWW + part * 4, baseA[h] + off);
 #pragma unroll
-    for (int h = 0; h < HB; ++h) cp_async16(sB + stage * BN * ROWW + ((tid + h * kThreads) >> 2) * ROWW + part * 4, baseB[h] + off);
+    for (int h = 0; h < HB; ++h) cp_async16(sB + stage * BN * ROWW + ((tid + h * kThreads) / PPR) * ROWW + part * 4, baseB[h] + off);
   };
 
   uint32_t acc[8][NJ];
@@ -362,10 +370,50 @@ static SadPlan choose_plan(int64_t nrows, int64_t S, int nkb, int sms) {
   return best;
 }
 
-template <bool kAtomic, bool kImage, int BN>
+template <bool kAtomic, bool kImage, int BN, int KW>
 static cudaError_t sad_set_attr() {
-  return cudaFuncSetAttribute(k_sad<kAtomic, kImage, BN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              sad::smem_bytes<BN>());
+  return cudaFuncSetAttribute(k_sad<kAtomic, kImage, BN, KW>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              sad::smem_bytes<BN, KW>());
+}
+template <int KW>
+static cudaError_t sad_set_attr_all() {
+  cudaError_t e;
+  if ((e = sad_set_attr<false, false, 128, KW>()) != cudaSuccess) return e;
+  if ((e = sad_set_attr<true, false, 128, KW>()) != cudaSuccess) return e;
+  if ((e = sad_set_attr<false, true, 128, KW>()) != cudaSuccess) return e;
+  if ((e = sad_set_attr<true, true, 128, KW>()) != cudaSuccess) return e;
+  if ((e = sad_set_attr<false, false, 64, KW>()) != cudaSuccess) return e;
+  if ((e = sad_set_attr<false, true, 64, KW>()) != cudaSuccess) return e;
+  if ((e = sad_set_attr<true, false, 64, KW>()) != cudaSuccess) return e;
+  return sad_set_attr<true, true, 64, KW>();
+}
+
+// One launch of the chosen plan for a stage width KW.
+template <int KW>
+static void sad_launch_kw(const SadGeom& g2, bool image, int bn, int split, int32_t nrows, int32_t S, int kw,
+                          int64_t gy, int32_t* E, int64_t ldE, int32_t* Ep, int64_t ldp, cudaStream_t st) {
+  using namespace sad;
+  if (bn == 64) {
+    dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, (unsigned)split);
+    constexpr int sm = smem_bytes<64, KW>();
+    if (split > 1) {
+      if (image) k_sad<true, true, 64, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
+      else k_sad<true, false, 64, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
+    } else {
+      if (image) k_sad<false, true, 64, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
+      else k_sad<false, false, 64, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
+    }
+  } else {
+    dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
+    constexpr int sm = smem_bytes<128, KW>();
+    if (split > 1) {   // (split-K accumulates: the sigma copy follows E, launch_sad_sigma)
+      if (image) k_sad<true, true, 128, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
+      else k_sad<true, false, 128, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
+    } else {
+      if (image) k_sad<false, true, 128, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
+      else k_sad<false, false, 128, KW><<<grid, kThreads, sm, st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
+    }
+  }
 }
 
 static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows, int32_t S, int32_t P,
@@ -379,18 +427,13 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
   static std::atomic<uint64_t> attr_done{0};   // one bit per device ordinal
   if (dev < 64 && !(attr_done.load() & (1ull << dev))) {
     cudaError_t e;
-    if ((e = sad_set_attr<false, false, 128>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<true, false, 128>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<false, true, 128>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<true, true, 128>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<false, false, 64>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<false, true, 64>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<true, false, 64>()) != cudaSuccess) return e;
-    if ((e = sad_set_attr<true, true, 64>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr_all<16>()) != cudaSuccess) return e;
+    if ((e = sad_set_attr_all<32>()) != cudaSuccess) return e;
     attr_done.fetch_or(1ull << dev);
   }
   const int kw = image ? P / 4 : (int)(geo.ldt / 4);
-  const int nkb = kw / BKW;
+  const int KWs = stage_words(kw);
+  const int nkb = kw / KWs;
   const int64_t gy = (nrows + BM - 1) / BM;
   if (gy > 65535) return cudaErrorInvalidValue;
   const SadPlan plan = choose_plan(nrows, S, nkb, sms);
@@ -406,26 +449,8 @@ static cudaError_t launch_sad_geom(const SadGeom& geo, bool image, int32_t nrows
         : cudaMemset2DAsync(E, sizeof(int32_t) * ldE, 0, sizeof(int32_t) * S, nrows, st);
     if (e != cudaSuccess) return e;
   }
-  if (plan.bn == 64) {
-    dim3 grid((unsigned)((S + 63) / 64), (unsigned)gy, (unsigned)split);
-    if (split > 1) {
-      if (image) k_sad<true, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
-      else k_sad<true, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
-    } else {
-      if (image) k_sad<false, true, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
-      else k_sad<false, false, 64><<<grid, kThreads, smem_bytes<64>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
-    }
-    note_launch();
-    return cudaGetLastError();
-  }
-  dim3 grid((unsigned)((S + 127) / 128), (unsigned)gy, (unsigned)split);
-  if (split > 1) {   // (split-K accumulates: the sigma copy follows E, launch_sad_sigma)
-    if (image) k_sad<true, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
-    else k_sad<true, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw / split, E, ldE, nullptr, 0);
-  } else {
-    if (image) k_sad<false, true, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
-    else k_sad<false, false, 128><<<grid, kThreads, smem_bytes<128>(), st>>>(g2, nrows, S, kw, E, ldE, Ep, ldp);
-  }
+  if (KWs == 32) sad_launch_kw<32>(g2, image, plan.bn, split, nrows, S, kw, gy, E, ldE, Ep, ldp, st);
+  else sad_launch_kw<16>(g2, image, plan.bn, split, nrows, S, kw, gy, E, ldE, Ep, ldp, st);
   note_launch();
   return cudaGetLastError();
 }
@@ -443,7 +468,7 @@ bool sad_split_plan(int32_t nrows, int32_t S, int32_t P) {
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  return choose_plan(nrows, S, (P / 4) / sad::BKW, sms).split > 1;
+  return choose_plan(nrows, S, (P / 4) / sad::stage_words(P / 4), sms).split > 1;
 }
 
 bool sad_image_ok(const uint8_t* I, const uint8_t* T, int32_t N, int32_t M, int32_t C) {
